@@ -1,0 +1,316 @@
+"""Benchmark: search-space points evaluated / s (and survivors / s) of the BEAST
+GEMM space enumeration on N B200s (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload NAME] [--impl reference]
+
+A step is one pass of the whole hot path: resolve,
+prefix stage L1-L7, flattener, A grids L8-L9, B grids L10-L11, compaction,
+write-out of every surviving record into device memory and, for N > 1, the
+combine (all_gather of counts -> offsets, all_reduce of the stats, gather of
+the survivors to rank 0 in canonical order).  value = N_canon (points of the
+canonical nest, every level) / device time per step,
+whole job, max over ranks.  The default workload is BASELINE.json configs[1],
+the paper's headline space (DGEMM, no transposes, K40c limits, default
+bounds).  Inputs are synthetic space descriptions (beast_inputs.py); there is
+no data.  --impl reference times the CPU oracle (oracle/, the only reference
+this paper-tier run has) on the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "search-space points evaluated/sec and survivors/sec at 1/2/4/8 B200"
+UNIT = "points/s"
+
+WORKLOADS = {
+    "headline": "BASELINE configs[1]: full 15-dimension DGEMM space, no transposes, Tesla K40c limits "
+                "(PAPER.md Figs 8-11), default bounds 1024, thresholds 256/2",
+    "b200_S": "BASELINE configs[3]: SGEMM NN with B200 (sm_100) limits, default bounds",
+    "b200_C": "BASELINE configs[3]: CGEMM NN with B200 (sm_100) limits, default bounds",
+    "b200_D": "BASELINE configs[3]: DGEMM NN with B200 (sm_100) limits, default bounds",
+    "widened256_b200": "BASELINE configs[4]: DGEMM NN, B200 limits, blk_m/blk_n/blk_k <= 256",
+    "widened256_k40c": "BASELINE configs[4]: DGEMM NN, K40c limits, blk_m/blk_n/blk_k <= 256",
+    "k40c_S": "BASELINE configs[2]: SGEMM NN, K40c limits",
+}
+
+# Paper timings of this path (context only):
+PAPER_CONTEXT = {"python_s": 66948, "c_s": 264, "cpu": "Xeon E5-2650 v3, 1 core"}
+
+
+def _load_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f), "measured"
+    except Exception:
+        return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}, "fallback"
+
+
+# ---------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index=0):
+        self.index = index
+        self.samples = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def start(self):
+        def run():
+            while not self._stop.is_set():
+                try:
+                    out = subprocess.run(["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.Q,
+                                          "--format=csv,noheader,nounits"], capture_output=True, text=True,
+                                         timeout=5).stdout.strip()
+                    if out:
+                        self.samples.append([x.strip() for x in out.split(",")])
+                except Exception:
+                    pass
+                self._stop.wait(0.1)
+        self._t = threading.Thread(target=run, daemon=True)
+        self._t.start()
+
+    def stop(self):
+        self._stop.set()
+        if self._t:
+            self._t.join(timeout=10)
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for s in self.samples:
+            for n, v in zip(names, s[4:8]):
+                if v.strip().lower() == "active":
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(self.samples)}
+
+
+# ---------------------------------------------------------------- reference arm
+def run_reference(args):
+    """CPU oracle (oracle/beast_oracle.c, OpenMP over dim_m) on the same
+    workload; each step enumerates the whole space (bounded: seconds)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import beast_inputs
+    import oracle
+    desc = beast_inputs.named(args.workload)
+    cores = os.cpu_count() or 1
+    n_canon = None
+    survivors = None
+    for _ in range(args.warmup):
+        r = oracle.nest(desc, threads=cores, digest=False)
+    times = []
+    for _ in range(args.steps):
+        t = time.perf_counter()
+        r = oracle.nest(desc, threads=cores, digest=False)
+        times.append(time.perf_counter() - t)
+        n_canon, survivors = sum(r["visits"]), r["survivors"]
+    ms = 1e3 * sum(times) / len(times)
+    value = n_canon / (ms / 1e3)
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+        "config": {"workload": args.workload, "description": WORKLOADS.get(args.workload, args.workload),
+                   "n_canon": n_canon, "survivors": survivors},
+        "survivors_per_s": survivors / (ms / 1e3),
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
+                         "sample": "whole %s space per step (%d points), canonical nest, OpenMP over dim_m"
+                                   % (args.workload, n_canon)},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ---------------------------------------------------------------- GPU arm
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--workload", default="headline", choices=sorted(WORKLOADS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+
+    import beast_inputs
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_ipps_luszczekgkdd16_b200 as beast
+    from paper_conf_ipps_luszczekgkdd16_b200 import dist as bdist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        world = args.gpus if world == 1 and args.gpus == 1 else world
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    desc = beast_inputs.named(args.workload)
+    sp = beast.Space.from_desc(desc)
+    stream = torch.cuda.current_stream()
+
+    # sizes (and the canonical point count) from one instrumented pass
+    _, st_local = sp.enumerate(rank=rank, world=world, stats=True)
+    stats = bdist.combine_stats(st_local, world)
+    n_canon = stats["points"]
+    survivors = stats["survivors"]
+
+    out = torch.empty((max(st_local["survivors"], 1), 2), dtype=torch.uint64, device="cuda")
+    gathered = torch.empty((max(survivors, 1), 2), dtype=torch.uint64, device="cuda") if rank == 0 else None
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")   # > 126 MB L2
+
+    def step():
+        n = beast.beast_enumerate(sp.handle, out, rank, world, stream)
+        if world > 1:
+            bdist.gather_records(out[:n], gathered, world)
+        return n
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+
+    sp.set_timing(True)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    a_eval_ms = []
+    launches = 0
+    clocks = ClockSampler(local)
+    clocks.start()
+    time.sleep(0.3)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    for i in range(args.steps):
+        flush.zero_()                     # L2 flush between timed steps (not timed)
+        ev[i][0].record(stream)
+        step()
+        ev[i][1].record(stream)
+        k, ams, _ = sp.last_launches()
+        launches += k
+        a_eval_ms.append(ams)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clocks.stop()
+    sp.set_timing(False)
+    total_ms = sum(a.elapsed_time(b) for a, b in ev)
+    if world > 1:
+        t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms = float(t.item())
+    ms = total_ms / args.steps
+
+    # e2e: the same metric through the public host-buffer call (list copied
+    # back to pinned host memory every step)
+    host = torch.empty((max(st_local["survivors"], 1), 2), dtype=torch.uint64).pin_memory()
+    for _ in range(2):
+        beast.beast_enumerate_to_host(sp.handle, host, rank, world, stream)
+    torch.cuda.synchronize()
+    e2e_ms = []
+    for _ in range(max(3, args.steps // 2)):
+        flush.zero_()
+        torch.cuda.synchronize()
+        t = time.perf_counter()
+        beast.beast_enumerate_to_host(sp.handle, host, rank, world, stream)
+        e2e_ms.append(1e3 * (time.perf_counter() - t))
+    e2e_step = statistics.median(e2e_ms)
+    if world > 1:
+        t = torch.tensor([e2e_step], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_step = float(t.item())
+
+    line = None
+    if rank == 0:
+        peaks, peak_src = _load_peaks()
+        a_ms = statistics.mean(a_eval_ms)
+        a_points = stats["visits"][8]          # L9 points: one launch evaluates all of them
+        ops_per_point = 2                      # one multiply-add forming dim_m_a*dim_n_a, one compare
+        sm_count = torch.cuda.get_device_properties(0).multi_processor_count
+        lanes = 128                            # int lanes / clk / SM: ALU pipe 64 + FMA pipe 64
+        peak_ops = sm_count * lanes * float(peaks.get("sm_max_mhz", 1965.0)) * 1e6
+        achieved = ops_per_point * a_points / (a_ms / 1e3) / world if a_ms > 0 else 0.0
+        traffic = None
+        prof = os.path.join(ROOT, "profiles", "k_eval_traffic.json")
+        if os.path.exists(prof):
+            try:
+                traffic = json.load(open(prof)).get(args.workload)
+            except Exception:
+                traffic = None
+        clk = clocks.summary()
+        cpu = None
+        if world == 1 and not args.no_cpu_baseline:
+            cpu = cpu_baseline(desc)
+        line = {
+            "metric": METRIC, "value": n_canon / (ms / 1e3), "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": args.workload, "description": WORKLOADS[args.workload],
+                       "n_canon": n_canon, "survivors": survivors,
+                       "l2": "flushed between timed steps (256 MiB write)", "parallelism": "dp%d" % world},
+            "survivors_per_s": survivors / (ms / 1e3),
+            "roofline": {"bound": "alu", "kernel": "k_eval<A> (L8-L9 A-read grids)",
+                         "achieved": achieved / 1e12, "peak": peak_ops / 1e12, "unit": "Tops/s",
+                         "frac": achieved / peak_ops if peak_ops else None, "traffic": traffic,
+                         "algorithmic_ops_per_launch": ops_per_point * a_points // world,
+                         "avg_launch_ms": a_ms,
+                         "peak_source": "%d SMs x %d int lanes/clk x sm_max_mhz (%s MEASURED_PEAKS.json)"
+                                        % (sm_count, lanes, peak_src)},
+            "e2e": {"value": n_canon / (e2e_step / 1e3), "unit": UNIT,
+                    "h2d_bytes_per_step": 96,
+                    "d2h_bytes_per_step": 16 * st_local["survivors"] + 512},
+            "gpu_launches": launches,
+            "clocks": clk,
+            "cpu_baseline": cpu,
+            "stages_ms": sp.last_stage_ms(),
+            "paper_context": PAPER_CONTEXT,
+        }
+        print(json.dumps(line), flush=True)
+    sp.close()
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+def cpu_baseline(desc):
+    import oracle
+    cores = os.cpu_count() or 1
+    t = time.perf_counter()
+    r = oracle.nest(desc, threads=cores, digest=False)
+    dt = time.perf_counter() - t
+    pts = sum(r["visits"])
+    return {"value": pts / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": "whole space once (%d points, %.1f s wall on %d threads), canonical nest" % (pts, dt, cores),
+            "survivors_per_s": r["survivors"] / dt}
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -154,6 +154,9 @@ int beast_abi_version(void);
 /* Human-readable text of a status code (static storage). */
 const char *beast_error_string(int status);
 
+/* Text of the last error recorded on this handle (empty if none). */
+const char *beast_last_error(const beast_space *space);
+
 /* Fig 8 values of a Tesla K40c with the Fig 9 fields resolved for
  * cc 3.5 (16 blocks, 64 warps, 255 registers).  out: caller-owned. */
 int beast_limits_k40c(beast_device_limits *out);

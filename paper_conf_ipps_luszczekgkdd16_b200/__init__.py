@@ -1,0 +1,234 @@
+"""B200-native BEAST GEMM search-space enumerator (Luszczek et al., IPDPSW 2016).
+
+Python face of include/beast.h.  The functions named beast_* mirror the C ABI
+one to one (argument marshalling only); `Space` is a small convenience
+wrapper over them.  All enumeration runs in libbeast.so on the GPU.
+
+    import beast_inputs, paper_conf_ipps_luszczekgkdd16_b200 as beast
+    sp = beast.Space.from_desc(beast_inputs.headline())
+    n = sp.count()                       # 1,207,600
+    rec = sp.enumerate()                 # torch.uint64 (n, 2) [lo, hi] on cuda
+"""
+from __future__ import annotations
+
+import ctypes
+
+from . import _lib
+from ._lib import (BEAST_ERR_CAPACITY, BEAST_OK, PRECISION, beast_bounds,  # noqa: F401
+                   beast_device_limits, beast_settings, beast_stats)
+
+STAT_PREDICATES = (
+    "over_max_threads", "over_max_regs_per_thread", "over_max_regs_per_block",
+    "over_max_shmem", "low_occupancy_regs", "low_occupancy_shmem", "low_fmas",
+    "partial_warps", "cant_reshape_a1", "cant_reshape_b1", "cant_reshape_a2",
+    "cant_reshape_b2",
+)
+
+
+class BeastError(RuntimeError):
+    def __init__(self, status, msg=""):
+        self.status = status
+        super().__init__("%s (%d)%s" % (_lib.lib().beast_error_string(status).decode(), status,
+                                        (": " + msg) if msg else ""))
+
+
+def _check(rc, handle=None):
+    if rc != BEAST_OK:
+        msg = _lib.lib().beast_last_error(handle).decode() if handle else ""
+        raise BeastError(rc, msg)
+
+
+def _stream_ptr(stream):
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream))
+
+
+# ----------------------------------------------------------- C-ABI mirrors
+def beast_abi_version() -> int:
+    return _lib.lib().beast_abi_version()
+
+
+def beast_limits_k40c() -> beast_device_limits:
+    out = beast_device_limits()
+    _check(_lib.lib().beast_limits_k40c(ctypes.byref(out)))
+    return out
+
+
+def beast_limits_from_device(device: int = 0) -> beast_device_limits:
+    out = beast_device_limits()
+    _check(_lib.lib().beast_limits_from_device(device, ctypes.byref(out)))
+    return out
+
+
+def beast_space_create(limits: beast_device_limits, precision, settings=None, bounds=None):
+    h = ctypes.c_void_p()
+    p = PRECISION[precision] if isinstance(precision, str) else int(precision)
+    _check(_lib.lib().beast_space_create(ctypes.byref(limits), p,
+                                         ctypes.byref(settings) if settings is not None else None,
+                                         ctypes.byref(bounds) if bounds is not None else None,
+                                         ctypes.byref(h)))
+    return h
+
+
+def beast_space_destroy(handle) -> None:
+    _lib.lib().beast_space_destroy(handle)
+
+
+def beast_count(handle, rank=0, world=1, stream=None, stats=False):
+    n = ctypes.c_uint64(0)
+    st = beast_stats() if stats else None
+    _check(_lib.lib().beast_count(handle, rank, world, _stream_ptr(stream), ctypes.byref(n),
+                                  ctypes.byref(st) if st is not None else None), handle)
+    return (int(n.value), stats_dict(st)) if stats else int(n.value)
+
+
+def beast_enumerate(handle, out, rank=0, world=1, stream=None, stats=False):
+    """out: torch.uint64 CUDA tensor of shape (capacity, 2), contiguous.
+    Returns the number of records written (and stats)."""
+    n = ctypes.c_uint64(0)
+    st = beast_stats() if stats else None
+    cap = out.shape[0] if out is not None else 0
+    ptr = ctypes.c_void_p(out.data_ptr()) if out is not None and cap else None
+    rc = _lib.lib().beast_enumerate(handle, rank, world, _stream_ptr(stream), ptr, cap,
+                                    ctypes.byref(n), ctypes.byref(st) if st is not None else None)
+    if rc == BEAST_ERR_CAPACITY:
+        raise BeastError(rc, "need %d records" % n.value)
+    _check(rc, handle)
+    return (int(n.value), stats_dict(st)) if stats else int(n.value)
+
+
+def beast_enumerate_to_host(handle, out, rank=0, world=1, stream=None, stats=False):
+    """out: pinned CPU torch.uint64 tensor (capacity, 2)."""
+    n = ctypes.c_uint64(0)
+    st = beast_stats() if stats else None
+    cap = out.shape[0] if out is not None else 0
+    ptr = ctypes.c_void_p(out.data_ptr()) if out is not None and cap else None
+    rc = _lib.lib().beast_enumerate_to_host(handle, rank, world, _stream_ptr(stream), ptr, cap,
+                                            ctypes.byref(n), ctypes.byref(st) if st is not None else None)
+    if rc == BEAST_ERR_CAPACITY:
+        raise BeastError(rc, "need %d records" % n.value)
+    _check(rc, handle)
+    return (int(n.value), stats_dict(st)) if stats else int(n.value)
+
+
+def beast_digest(records, base=0, stream=None) -> int:
+    """Digest of a CUDA uint64 (n, 2) [lo, hi] record tensor."""
+    d = ctypes.c_uint64(0)
+    n = records.shape[0]
+    _check(_lib.lib().beast_digest(ctypes.c_void_p(records.data_ptr()) if n else None, n, base,
+                                   _stream_ptr(stream), ctypes.byref(d)))
+    return int(d.value)
+
+
+def stats_dict(st: beast_stats) -> dict:
+    return dict(visits=[int(x) for x in st.visits], rejected=[int(x) for x in st.rejected],
+                survivors=int(st.survivors), prefixes=int(st.prefixes),
+                valid_a=int(st.valid_a), tuples=int(st.tuples),
+                points=int(sum(st.visits)))
+
+
+# ----------------------------------------------------------- convenience
+def limits_from_desc(desc: dict) -> beast_device_limits:
+    return beast_device_limits(*[int(desc.get(f, 0)) for f, _ in beast_device_limits._fields_])
+
+
+class Space:
+    """Owns one beast_space handle; scratch comes from torch's caching
+    allocator on the current device."""
+
+    def __init__(self, limits: beast_device_limits, precision, settings=None, bounds=None,
+                 torch_alloc: bool = True):
+        self.handle = beast_space_create(limits, precision, settings, bounds)
+        self._cb = None
+        if torch_alloc:
+            self._install_torch_allocator()
+
+    @classmethod
+    def from_desc(cls, desc: dict, **kw):
+        """desc: a beast_inputs space description."""
+        s = beast_settings(desc["trans_a"], desc["trans_b"],
+                           desc["min_threads_per_multi_processor"], desc["min_fmas_per_load"])
+        b = beast_bounds(desc["dim_m_max"], desc["dim_n_max"], desc["blk_m_max"],
+                         desc["blk_n_max"], desc["blk_k_max"])
+        return cls(limits_from_desc(desc), desc["precision"], s, b, **kw)
+
+    def _install_torch_allocator(self):
+        import torch
+        dev = torch.cuda.current_device()
+
+        def _alloc(nbytes, stream, ctx):
+            try:
+                return torch.cuda.caching_allocator_alloc(int(nbytes), dev, stream or 0)
+            except Exception:
+                return None
+
+        def _free(ptr, nbytes, stream, ctx):
+            torch.cuda.caching_allocator_delete(ptr)
+
+        self._cb = (_lib.ALLOC_FN(_alloc), _lib.FREE_FN(_free))
+        _check(_lib.lib().beast_space_set_allocator(self.handle, self._cb[0], self._cb[1], None))
+
+    def resolved(self) -> dict:
+        lim, st, bd = beast_device_limits(), beast_settings(), beast_bounds()
+        _check(_lib.lib().beast_space_resolved(self.handle, ctypes.byref(lim), ctypes.byref(st),
+                                               ctypes.byref(bd)))
+        d = {f: getattr(lim, f) for f, _ in lim._fields_}
+        d.update({f: getattr(st, f) for f, _ in st._fields_})
+        d.update({f: getattr(bd, f) for f, _ in bd._fields_})
+        return d
+
+    def count(self, rank=0, world=1, stream=None, stats=False):
+        return beast_count(self.handle, rank, world, stream, stats)
+
+    def enumerate(self, rank=0, world=1, stream=None, stats=False, out=None):
+        """Returns the shard's records as a CUDA uint64 tensor (n, 2) [lo, hi]
+        (a view of `out` if given), plus stats if requested."""
+        import torch
+        if out is None:
+            n = self.count(rank, world, stream)
+            out = torch.empty((max(n, 1), 2), dtype=torch.uint64, device="cuda")
+        r = beast_enumerate(self.handle, out, rank, world, stream, stats)
+        n = r[0] if stats else r
+        return (out[:n], r[1]) if stats else out[:n]
+
+    def set_timing(self, enable=True):
+        _check(_lib.lib().beast_space_set_timing(self.handle, int(enable)))
+
+    def last_stage_ms(self):
+        ms = (ctypes.c_float * 5)()
+        _check(_lib.lib().beast_last_stage_ms(self.handle, ms))
+        return list(ms)
+
+    def last_launches(self):
+        k, ms, n = ctypes.c_uint64(0), ctypes.c_float(0), ctypes.c_uint64(0)
+        _check(_lib.lib().beast_last_launches(self.handle, ctypes.byref(k), ctypes.byref(ms),
+                                              ctypes.byref(n)))
+        return int(k.value), float(ms.value), int(n.value)
+
+    def close(self):
+        if self.handle:
+            beast_space_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+
+def unpack(lo: int, hi: int) -> tuple:
+    """15-tuple of a packed record (include/beast.h layout)."""
+    lo, hi = int(lo), int(hi)
+    m = 0xFFF
+    return ((hi >> 52) & m, (hi >> 40) & m, (hi >> 28) & m, (hi >> 16) & m, (hi >> 4) & m,
+            (hi >> 1) & 7, hi & 1, (lo >> 52) & m, (lo >> 40) & m, (lo >> 28) & m,
+            (lo >> 16) & m, (lo >> 3) & 1, (lo >> 2) & 1, (lo >> 1) & 1, lo & 1)

@@ -1,0 +1,121 @@
+"""Multi-GPU combine (§X-B: parallelise the
+outermost loop nests).
+
+One process per GPU (torchrun).  Every rank runs the replicated prefix stage
+and enumerates its own contiguous canonical shard of L7 prefixes through the
+C ABI (beast_enumerate(rank, world)); the library never communicates.  This
+module does the one exchange the method has:
+
+  all_gather of the per-rank survivor counts -> exclusive scan = each shard's
+  global offset; all_reduce(sum) of the statistics; gather of the survivor
+  records to rank 0 in rank order (= canonical order), with point-to-point
+  transfers into rank 0's buffer at the scanned offsets (NCCL over NVLink on
+  GPUs, gloo in the CPU tests).
+
+The functions take and return torch tensors on whatever device the process
+group uses; they contain no enumeration logic.
+"""
+from __future__ import annotations
+
+import torch
+import torch.distributed as dist
+
+STAT_LEN = 15 + 12 + 4   # visits, rejected, survivors, prefixes, valid_a, tuples
+
+
+def _dev():
+    return torch.device("cuda", torch.cuda.current_device()) \
+        if dist.is_initialized() and dist.get_backend() == "nccl" else torch.device("cpu")
+
+
+def stats_to_tensor(st: dict, device=None) -> torch.Tensor:
+    v = list(st["visits"]) + list(st["rejected"]) + [st["survivors"], st["prefixes"], st["valid_a"], st["tuples"]]
+    return torch.tensor(v, dtype=torch.int64, device=device or _dev())
+
+
+def tensor_to_stats(t: torch.Tensor) -> dict:
+    v = [int(x) for x in t.cpu().tolist()]
+    st = dict(visits=v[:15], rejected=v[15:27], survivors=v[27], prefixes=v[28], valid_a=v[29], tuples=v[30])
+    st["points"] = sum(st["visits"])
+    return st
+
+
+def combine_stats(st: dict, world: int) -> dict:
+    """Sum the per-shard statistics over all ranks (each level L1..L6 is
+    charged to rank 0 only by the library, so the sum is the whole space)."""
+    if world <= 1 or not dist.is_initialized():
+        out = dict(st)
+        out["points"] = sum(st["visits"])
+        return out
+    t = stats_to_tensor(st)
+    dist.all_reduce(t, op=dist.ReduceOp.SUM)
+    return tensor_to_stats(t)
+
+
+def shard_offsets(n_local: int, world: int, device=None) -> list:
+    """all_gather of the shard sizes; returns [offset_0, ..., offset_world]
+    (exclusive scan, offset_world = total)."""
+    if world <= 1 or not dist.is_initialized():
+        return [0, n_local]
+    dev = device or _dev()
+    mine = torch.tensor([n_local], dtype=torch.int64, device=dev)
+    allc = [torch.zeros(1, dtype=torch.int64, device=dev) for _ in range(world)]
+    dist.all_gather(allc, mine)
+    counts = [int(c.item()) for c in allc]
+    offs = [0]
+    for c in counts:
+        offs.append(offs[-1] + c)
+    return offs
+
+
+def gather_records(local: torch.Tensor, gathered, world: int, root: int = 0) -> int:
+    """Gather every rank's (n_r, 2) record shard into `gathered` on `root` at
+    its canonical offset.  Returns the global count (on every rank)."""
+    n = int(local.shape[0])
+    offs = shard_offsets(n, world, local.device)
+    total = offs[-1]
+    if world <= 1 or not dist.is_initialized():
+        if gathered is not None and gathered.data_ptr() != local.data_ptr() and n:
+            gathered[:n].copy_(local)
+        return total
+    rank = dist.get_rank()
+    lv = local.view(torch.int64) if local.dtype == torch.uint64 else local
+    ops = []
+    if rank == root:
+        gv = gathered.view(torch.int64) if gathered.dtype == torch.uint64 else gathered
+        for r in range(world):
+            a, b = offs[r], offs[r + 1]
+            if b == a:
+                continue
+            if r == root:
+                gv[a:b].copy_(lv)
+            else:
+                ops.append(dist.P2POp(dist.irecv, gv[a:b], r))
+    elif n:
+        ops.append(dist.P2POp(dist.isend, lv.contiguous(), root))
+    if ops:
+        for req in dist.batch_isend_irecv(ops):
+            req.wait()
+    return total
+
+
+def enumerate_distributed(space, gather=False, stats=False, stream=None) -> dict:
+    """Enumerate this rank's shard with the library and combine.  Every rank
+    must pass the same `gather`.  Returns dict(local=records of this shard,
+    offset=its global offset, total=global count, gathered=the full canonical
+    list on rank 0 when gather=True, stats=summed stats when stats=True)."""
+    world = dist.get_world_size() if dist.is_initialized() else 1
+    rank = dist.get_rank() if dist.is_initialized() else 0
+    if stats:
+        rec, st = space.enumerate(rank=rank, world=world, stream=stream, stats=True)
+    else:
+        rec, st = space.enumerate(rank=rank, world=world, stream=stream), None
+    offs = shard_offsets(int(rec.shape[0]), world, rec.device)
+    out = dict(local=rec, offset=offs[rank], total=offs[-1], gathered=None)
+    if gather:
+        buf = torch.empty((max(offs[-1], 1), 2), dtype=rec.dtype, device=rec.device) if rank == 0 else None
+        gather_records(rec, buf, world)
+        out["gathered"] = buf[:offs[-1]] if buf is not None else None
+    if stats:
+        out["stats"] = combine_stats(st, world)
+    return out

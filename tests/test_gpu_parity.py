@@ -1,0 +1,211 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle.
+
+Bar: integer work, so bit-exact — survivor count,
+canonically ordered packed list (memcmp or the order-sensitive digest),
+per-level visits and first-failing rejection counts.  Small spaces run the
+oracle here; full-size spaces compare with tests/golden/expected.json, which
+scripts/make_golden.py wrote from the oracle alone.
+"""
+from __future__ import annotations
+
+import os
+import random
+
+import numpy as np
+import pytest
+
+import beast_inputs as bi
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def beast():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.fail("CUDA device required for -m gpu tests")
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_ipps_luszczekgkdd16_b200 as b
+    return b
+
+
+def _oracle_lohi(rec):
+    return np.stack([rec[:, 1], rec[:, 0]], axis=1) if len(rec) else np.zeros((0, 2), np.uint64)
+
+
+def _run(beast, desc, rank=0, world=1, stats=True):
+    with beast.Space.from_desc(desc) as sp:
+        rec, st = sp.enumerate(rank=rank, world=world, stats=True)
+        got = rec.cpu().numpy().copy()
+        dig = beast.beast_digest(rec) if len(rec) else 0
+        n = sp.count(rank=rank, world=world)
+    return got, st, dig, n
+
+
+def _check_small(beast, desc):
+    got, st, dig, n = _run(beast, desc)
+    ref = oracle.nest(desc, records=True)
+    want = _oracle_lohi(ref["records"])
+    assert got.shape == want.shape, (got.shape, want.shape)
+    assert np.array_equal(got, want)
+    assert n == ref["survivors"] == st["survivors"]
+    assert st["visits"] == ref["visits"], (st["visits"], ref["visits"])
+    assert st["rejected"] == ref["rejected"], (st["rejected"], ref["rejected"])
+    if len(got):
+        assert dig == ref["digest"]
+
+
+@pytest.mark.parametrize("p", bi.PRECISIONS)
+@pytest.mark.parametrize("ta,tb", bi.TRANSPOSES)
+def test_tiny(beast, p, ta, tb):
+    _check_small(beast, bi.tiny(p, ta, tb))
+
+
+def test_micro(beast):
+    _check_small(beast, bi.micro("C"))
+
+
+@pytest.mark.parametrize("seed", range(200))
+def test_fuzz(beast, seed):
+    _check_small(beast, bi.fuzz_space(seed))
+
+
+def test_empty_space(beast):
+    # warp_size larger than any threads_per_block: L2 rejects everything
+    desc = bi.make_space(dict(bi.K40C_DEVICE, max_threads_per_block=16), "D", bounds=8)
+    got, st, dig, n = _run(beast, desc)
+    assert n == 0 and got.shape == (0, 2) and st["survivors"] == 0
+    _check_small(beast, desc)
+
+
+def test_degenerate_bounds_one(beast):
+    _check_small(beast, bi.make_space(bi.K40C_DEVICE, "S", bounds=1))
+    _check_small(beast, bi.make_space(dict(bi.K40C_DEVICE, warp_size=1), "S", bounds=1))
+
+
+def test_headline_bit_exact(beast):
+    desc = bi.headline()
+    got, st, dig, n = _run(beast, desc)
+    ref = oracle.nest(desc, threads=os.cpu_count(), records=True)
+    assert np.array_equal(got, _oracle_lohi(ref["records"]))
+    assert st["visits"] == ref["visits"] and st["rejected"] == ref["rejected"]
+    assert dig == ref["digest"] and n == 1_207_600
+
+
+GOLDEN_BIG = ["k40c_%s_%d%d" % (p, a, b) for p in bi.PRECISIONS for a, b in bi.TRANSPOSES] + \
+             ["b200_%s_%d%d" % (p, a, b) for p in bi.PRECISIONS for a, b in bi.TRANSPOSES] + \
+             ["widened%d_%s_D_00" % (w, d) for w in (64, 256, 512) for d in ("k40c", "b200")] + \
+             ["b200_48k_D_00", "b200_48k_S_00"]
+
+
+@pytest.mark.parametrize("key", GOLDEN_BIG)
+def test_full_size_vs_golden(beast, golden_expected, key):
+    if key not in golden_expected:
+        pytest.skip("golden not generated for " + key)
+    e = golden_expected[key]
+    import torch
+    with beast.Space.from_desc(e["space"]) as sp:
+        rec, st = sp.enumerate(stats=True)
+        assert st["survivors"] == e["survivors"]
+        assert st["visits"] == e["visits"], key
+        assert st["rejected"] == e["rejected"], key
+        assert "0x%016x" % beast.beast_digest(rec) == e["digest"], key
+        if e["first"]:
+            lo, hi = rec[0].cpu().numpy(), rec[-1].cpu().numpy()
+            assert ["%016x" % lo[1], "%016x" % lo[0]] == e["first"]
+            assert ["%016x" % hi[1], "%016x" % hi[0]] == e["last"]
+        # strictly increasing as u128 (canonical and unique), on the device
+        if len(rec) > 1:
+            a = rec.view(torch.int64)
+            hi_, lo_ = a[:, 1], a[:, 0]
+            # unsigned compare via sign flip
+            f = torch.tensor(-(1 << 63), dtype=torch.int64, device=a.device)
+            h0, h1 = hi_[:-1] ^ f, hi_[1:] ^ f
+            l0, l1 = lo_[:-1] ^ f, lo_[1:] ^ f
+            inc = (h0 < h1) | ((h0 == h1) & (l0 < l1))
+            assert bool(inc.all())
+        # sampled records satisfy all 12 predicates (oracle's evaluator)
+        idx = random.Random(1).sample(range(len(rec)), min(300, len(rec)))
+        host = rec.view(torch.int64)[idx].cpu().numpy().view(np.uint64) if idx else []
+        for lo_v, hi_v in host:
+            _, pred = oracle.point(e["space"], oracle.unpack(int(hi_v), int(lo_v)))
+            assert not any(pred.values())
+        assert sp.count() == e["survivors"]
+
+
+@pytest.mark.parametrize("world", [2, 3, 8])
+def test_virtual_ranks_concatenate(beast, world):
+    """Shards (rank, world) concatenated in rank order equal the world=1 list;
+    their stats sum to the whole space's."""
+    desc = bi.headline()
+    full, stf, _, _ = _run(beast, desc)
+    parts, visits, rejected = [], np.zeros(15, np.int64), np.zeros(12, np.int64)
+    for r in range(world):
+        got, st, _, _ = _run(beast, desc, rank=r, world=world)
+        parts.append(got)
+        visits += np.array(st["visits"], np.int64)
+        rejected += np.array(st["rejected"], np.int64)
+    cat = np.concatenate(parts)
+    assert np.array_equal(cat, full)
+    assert list(visits) == stf["visits"] and list(rejected) == stf["rejected"]
+
+
+def test_digest_is_additive_over_shards(beast):
+    import torch
+    desc = bi.tiny("C")
+    with beast.Space.from_desc(desc) as sp:
+        rec = sp.enumerate()
+        full = beast.beast_digest(rec)
+        k = 1000
+        assert (beast.beast_digest(rec[:k]) + beast.beast_digest(rec[k:].contiguous(), base=k)) % (1 << 64) == full
+        host = rec.cpu().numpy()
+        assert full == oracle.digest(np.stack([host[:, 1], host[:, 0]], 1))
+        del torch
+
+
+def test_capacity_error_reports_required(beast):
+    import torch
+    with beast.Space.from_desc(bi.tiny("D")) as sp:
+        small = torch.empty((10, 2), dtype=torch.uint64, device="cuda")
+        with pytest.raises(beast.BeastError) as e:
+            beast.beast_enumerate(sp.handle, small)
+        assert e.value.status == beast.BEAST_ERR_CAPACITY and "1824" in str(e.value)
+
+
+def test_enumerate_to_host_matches_device(beast):
+    import torch
+    desc = bi.headline()
+    with beast.Space.from_desc(desc) as sp:
+        dev = sp.enumerate().cpu().numpy()
+        host = torch.empty((dev.shape[0], 2), dtype=torch.uint64).pin_memory()
+        n = beast.beast_enumerate_to_host(sp.handle, host)
+        assert n == dev.shape[0]
+        assert np.array_equal(host.numpy(), dev)
+
+
+def test_stats_mode_does_not_change_results(beast):
+    desc = bi.k40c("Z")
+    with beast.Space.from_desc(desc) as sp:
+        a = sp.enumerate().cpu().numpy()
+        b, _ = sp.enumerate(stats=True)
+        assert np.array_equal(a, b.cpu().numpy())
+
+
+def test_repeated_calls_are_deterministic(beast):
+    desc = bi.headline()
+    with beast.Space.from_desc(desc) as sp:
+        a = beast.beast_digest(sp.enumerate())
+        for _ in range(3):
+            assert beast.beast_digest(sp.enumerate()) == a
+
+
+def test_limits_from_device_b200(beast):
+    lim = beast.beast_limits_from_device(0)
+    assert lim.cuda_major == 10 and lim.cuda_minor == 0
+    for k in ("max_threads_per_block", "max_threads_dim_x", "max_threads_dim_y", "warp_size",
+              "max_regs_per_block", "max_registers_per_multi_processor", "float_size",
+              "max_shared_mem_per_block", "max_shmem_per_multi_processor"):
+        assert getattr(lim, k) == bi.B200_DEVICE[k], (k, getattr(lim, k))
+    assert lim.max_blocks_per_multi_processor == 32 and lim.max_registers_per_thread == 255
