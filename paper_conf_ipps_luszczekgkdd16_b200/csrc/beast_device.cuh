@@ -91,44 +91,6 @@ __device__ __forceinline__ void st_volatile_u64(uint64_t *p, uint64_t v) {
     asm volatile("st.volatile.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-// --------------------------------------------- decoupled look-back prefix
-// Tile status word: [63:62] flag (0 empty, 1 aggregate, 2 inclusive prefix),
-// [61:0] value.  Tiles are handed out in increasing order by an atomic
-// counter, so every predecessor of a tile is owned by a resident CTA and the
-// look-back always terminates.
-constexpr uint64_t kFlagAgg = 1ull << 62;
-constexpr uint64_t kFlagInc = 2ull << 62;
-constexpr uint64_t kValMask = (1ull << 62) - 1;
-
-// Called by ALL 32 lanes of one warp.  Publishes `aggregate` for `tile` and
-// returns the exclusive prefix of all earlier tiles.
-__device__ __forceinline__ uint64_t lookback_exclusive(uint64_t *status, uint64_t tile,
-                                                       uint64_t aggregate) {
-    const uint32_t lane = lane_id();
-    if (tile == 0) {
-        if (lane == 0) st_volatile_u64(&status[0], kFlagInc | aggregate);
-        return 0;
-    }
-    if (lane == 0) st_volatile_u64(&status[tile], kFlagAgg | aggregate);
-    uint64_t exclusive = 0;
-    int64_t base = (int64_t)tile - 1;
-    while (true) {
-        const int64_t t = base - (int64_t)lane;
-        uint64_t s = t >= 0 ? ld_volatile_u64(&status[t]) : kFlagInc;
-        while (__any_sync(kFull, (s >> 62) == 0)) {
-            if ((s >> 62) == 0) s = ld_volatile_u64(&status[t]);
-        }
-        const uint32_t inc = __ballot_sync(kFull, (s >> 62) == 2);
-        const int stop = inc ? __ffs(inc) - 1 : 32;
-        const uint64_t v = (int)lane <= stop ? (s & kValMask) : 0;
-        exclusive += warp_sum_u64(v);
-        if (inc) break;
-        base -= 32;
-    }
-    if (lane == 0) st_volatile_u64(&status[tile], kFlagInc | (exclusive + aggregate));
-    return exclusive;
-}
-
 // Exclusive scan of one u32 per thread over a CTA of NT threads.
 // Returns the thread's exclusive prefix; *total receives the CTA sum.
 template <int NT>
@@ -187,51 +149,61 @@ __device__ __forceinline__ uint64_t cta_exclusive_scan64(uint64_t v, uint64_t *s
 }
 
 // --------------------------------------------------- the hot inner loop
-// Evaluates cant_reshape_{a,b}1, "dim_m_x * dim_n_x !=
-// threads_per_block", on 16 consecutive points of one grid row: the row
-// holds the short-axis coordinate `s` fixed and runs the long-axis
-// coordinate over base/s + 1 .. base/s + 16, so the products are
-// base + s*1 .. base + s*16.  One IMAD (FMA pipe) forms each product and one
-// ISETP.EQ.OR (ALU pipe) compares it with T and folds it into the row's hit
-// predicate: two issue slots per point, the two pipes evenly loaded.
-__device__ __forceinline__ uint32_t eval16(uint32_t hit, uint32_t base, uint32_t s, uint32_t T) {
+// cant_reshape_a1 / b1: "dim_m_x * dim_n_x != threads_per_block".
+// A grid row holds its short-axis coordinate s fixed while the long-axis
+// coordinate j runs 1..L, so the row's points are the products s*j, j <= L.
+//
+// Two points per 32-bit lane: with J = j1 | j2 << 16 (j2 = j1 + 1) and
+// C = (2^16 - T) * 0x10001, the word s*J + C (mod 2^32) holds
+// (s*j1 - T) mod 2^16 in its low half and (s*j2 - T) mod 2^16 in its high half
+// whenever s*j1 < T (no carry reaches the high half) — in particular whenever
+// s*j2 == T.  So a point with s*j == T always leaves a zero half (no false
+// negatives); a zero half can also come from s*j == T (mod 2^16) with
+// s*j != T, which the exact check after the loop rejects.  One IMAD or IADD
+// forms a pair, and ptxas fuses two min.u16x2 into one VIMNMX3.U16x2 that
+// folds two pairs into the row's running minimum: 16 points cost 8 product
+// instructions + 4 min instructions.
+__device__ __forceinline__ uint32_t eval16p(uint32_t acc, uint32_t C, uint32_t s, uint32_t d2) {
     asm volatile(
-        "{\n\t.reg .pred p;\n\t.reg .u32 t<16>;\n\t"
-        "setp.ne.u32 p, %0, 0;\n\t"
-        "mad.lo.u32 t0, %2, 1, %1;\n\t setp.eq.or.u32 p, t0, %3, p;\n\t"
-        "mad.lo.u32 t1, %2, 2, %1;\n\t setp.eq.or.u32 p, t1, %3, p;\n\t"
-        "mad.lo.u32 t2, %2, 3, %1;\n\t setp.eq.or.u32 p, t2, %3, p;\n\t"
-        "mad.lo.u32 t3, %2, 4, %1;\n\t setp.eq.or.u32 p, t3, %3, p;\n\t"
-        "mad.lo.u32 t4, %2, 5, %1;\n\t setp.eq.or.u32 p, t4, %3, p;\n\t"
-        "mad.lo.u32 t5, %2, 6, %1;\n\t setp.eq.or.u32 p, t5, %3, p;\n\t"
-        "mad.lo.u32 t6, %2, 7, %1;\n\t setp.eq.or.u32 p, t6, %3, p;\n\t"
-        "mad.lo.u32 t7, %2, 8, %1;\n\t setp.eq.or.u32 p, t7, %3, p;\n\t"
-        "mad.lo.u32 t8, %2, 9, %1;\n\t setp.eq.or.u32 p, t8, %3, p;\n\t"
-        "mad.lo.u32 t9, %2, 10, %1;\n\t setp.eq.or.u32 p, t9, %3, p;\n\t"
-        "mad.lo.u32 t10, %2, 11, %1;\n\t setp.eq.or.u32 p, t10, %3, p;\n\t"
-        "mad.lo.u32 t11, %2, 12, %1;\n\t setp.eq.or.u32 p, t11, %3, p;\n\t"
-        "mad.lo.u32 t12, %2, 13, %1;\n\t setp.eq.or.u32 p, t12, %3, p;\n\t"
-        "mad.lo.u32 t13, %2, 14, %1;\n\t setp.eq.or.u32 p, t13, %3, p;\n\t"
-        "mad.lo.u32 t14, %2, 15, %1;\n\t setp.eq.or.u32 p, t14, %3, p;\n\t"
-        "mad.lo.u32 t15, %2, 16, %1;\n\t setp.eq.or.u32 p, t15, %3, p;\n\t"
-        "selp.u32 %0, 1, 0, p;\n\t}"
-        : "+r"(hit)
-        : "r"(base), "r"(s), "r"(T));
-    return hit;
+        "{\n\t.reg .b32 t<8>;\n\t"
+        "mad.lo.u32 t0, %2, 0x00020001, %1;\n\t"
+        "add.u32 t1, t0, %3;\n\t"
+        "min.u16x2 %0, %0, t0;\n\t min.u16x2 %0, %0, t1;\n\t"
+        "mad.lo.u32 t2, %2, 0x00060005, %1;\n\t"
+        "mad.lo.u32 t3, %2, 0x00080007, %1;\n\t"
+        "min.u16x2 %0, %0, t2;\n\t min.u16x2 %0, %0, t3;\n\t"
+        "mad.lo.u32 t4, %2, 0x000a0009, %1;\n\t"
+        "add.u32 t5, t4, %3;\n\t"
+        "min.u16x2 %0, %0, t4;\n\t min.u16x2 %0, %0, t5;\n\t"
+        "mad.lo.u32 t6, %2, 0x000e000d, %1;\n\t"
+        "mad.lo.u32 t7, %2, 0x0010000f, %1;\n\t"
+        "min.u16x2 %0, %0, t6;\n\t min.u16x2 %0, %0, t7;\n\t"
+        "}"
+        : "+r"(acc)
+        : "r"(C), "r"(s), "r"(d2));
+    return acc;
 }
 
-// Whole row of L points: products s*1 .. s*L compared with T.
+// Whole row: the points s*1 .. s*L against T (T <= 65535, s, L <= 4095).
+// The loop runs ceil(L/16) blocks; products past L are computed but a match
+// there is rejected by the exact check (j = T/s must satisfy j <= L).
+// Returns the unique j in [1, L] with s*j == T, or 0.  s == 0 marks an idle
+// lane.  T/s is formed with the fp32 reciprocal: for T < 2^16 and s < 2^12
+// its error is far below 1/2, so rounding gives the exact quotient whenever
+// s divides T, and the integer check s*j == T decides.
 __device__ __forceinline__ uint32_t eval_row(uint32_t s, uint32_t T, uint32_t L) {
-    uint32_t hit = 0, base = 0, j = 0;
-    for (; j + 16 <= L; j += 16) {
-        hit = eval16(hit, base, s, T);
-        base += 16u * s;
+    uint32_t C = (0x10000u - T) * 0x10001u;
+    const uint32_t step = s * 0x00100010u;   // +16 on each half's index
+    const uint32_t d2 = s * 0x00020002u;     // +2 on each half's index
+    uint32_t acc = 0xffffffffu;
+    for (uint32_t j = 0; j < L; j += 16) {
+        acc = eval16p(acc, C, s, d2);
+        C += step;
     }
-    for (; j < L; ++j) {
-        base += s;
-        hit |= (base == T);
-    }
-    return hit;
+    const bool cand = s != 0 && ((acc & 0xffffu) == 0 || (acc >> 16) == 0);
+    if (!cand) return 0;
+    const uint32_t t = __float2uint_rn(__fdividef((float)T, (float)s));
+    return (t * s == T && t <= L) ? t : 0u;
 }
 
 }  // namespace beast
