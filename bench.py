@@ -57,30 +57,46 @@ def _load_peaks():
 
 # ---------------------------------------------------------------- clocks
 class ClockSampler:
-    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    """SM clock and throttle reasons sampled through NVML every 10 ms during
+    the timed region (falls back to nvidia-smi if NVML is unavailable)."""
 
-    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
-         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    REASONS = {  # NVML clocks-event reason bits
+        0x8: "hw_slowdown", 0x40: "hw_thermal_slowdown", 0x20: "sw_thermal_slowdown",
+        0x4: "sw_power_cap", 0x80: "hw_power_brake_slowdown",
+    }
 
     def __init__(self, index=0):
         self.index = index
-        self.samples = []
+        self.sm, self.sm_max, self.reasons = [], None, set()
         self._stop = threading.Event()
         self._t = None
 
     def start(self):
         def run():
-            while not self._stop.is_set():
-                try:
-                    out = subprocess.run(["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.Q,
-                                          "--format=csv,noheader,nounits"], capture_output=True, text=True,
-                                         timeout=5).stdout.strip()
-                    if out:
-                        self.samples.append([x.strip() for x in out.split(",")])
-                except Exception:
-                    pass
-                self._stop.wait(0.1)
+            try:
+                import pynvml
+                pynvml.nvmlInit()
+                h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+                self.sm_max = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+                while not self._stop.is_set():
+                    self.sm.append(pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM))
+                    r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
+                    for bit, name in self.REASONS.items():
+                        if r & bit:
+                            self.reasons.add(name)
+                    self._stop.wait(0.01)
+            except Exception:
+                while not self._stop.is_set():
+                    try:
+                        out = subprocess.run(["nvidia-smi", "-i", str(self.index),
+                                              "--query-gpu=clocks.sm,clocks.max.sm", "--format=csv,noheader,nounits"],
+                                             capture_output=True, text=True, timeout=5).stdout.strip()
+                        a, b = [float(x) for x in out.split(",")]
+                        self.sm.append(a)
+                        self.sm_max = b
+                    except Exception:
+                        pass
+                    self._stop.wait(0.1)
         self._t = threading.Thread(target=run, daemon=True)
         self._t.start()
 
@@ -90,18 +106,10 @@ class ClockSampler:
             self._t.join(timeout=10)
 
     def summary(self):
-        if not self.samples:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
-        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
-        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = set()
-        for s in self.samples:
-            for n, v in zip(names, s[4:8]):
-                if v.strip().lower() == "active":
-                    reasons.add(n)
-        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": sorted(reasons), "samples": len(self.samples)}
+        if not self.sm:
+            return {"sm_mhz": None, "sm_max_mhz": self.sm_max, "reasons": ["unsampled"]}
+        return {"sm_mhz": statistics.median(self.sm), "sm_max_mhz": self.sm_max,
+                "reasons": sorted(self.reasons), "samples": len(self.sm)}
 
 
 # ---------------------------------------------------------------- reference arm
@@ -115,9 +123,22 @@ def run_reference(args):
     import oracle
     desc = beast_inputs.named(args.workload)
     cores = os.cpu_count() or 1
+    # Bounded sample: if the whole space per step would make the run longer
+    # than ~150 s on this host, each step enumerates the canonical prefix
+    # dim_m <= D of the same space (the first L1 values, all inner loops).
+    t = time.perf_counter()
+    r = oracle.nest(desc, threads=cores, digest=False)
+    full_t = time.perf_counter() - t
+    sample = "whole %s space per step" % args.workload
+    if full_t * (args.steps + args.warmup) > 150.0:
+        dmx = oracle.resolve(desc)["dim_m_max"]
+        frac = 150.0 / (full_t * (args.steps + args.warmup))
+        d = max(1, int(dmx * frac))
+        desc = dict(desc, dim_m_max=d)
+        sample = "canonical prefix dim_m <= %d of the %s space per step" % (d, args.workload)
     n_canon = None
     survivors = None
-    for _ in range(args.warmup):
+    for _ in range(args.warmup - 1):
         r = oracle.nest(desc, threads=cores, digest=False)
     times = []
     for _ in range(args.steps):
@@ -135,8 +156,7 @@ def run_reference(args):
                    "n_canon": n_canon, "survivors": survivors},
         "survivors_per_s": survivors / (ms / 1e3),
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
-                         "sample": "whole %s space per step (%d points), canonical nest, OpenMP over dim_m"
-                                   % (args.workload, n_canon)},
+                         "sample": "%s (%d points), canonical nest, OpenMP over dim_m" % (sample, n_canon)},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -147,8 +167,8 @@ def run_reference(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20)
-    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--workload", default="headline", choices=sorted(WORKLOADS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -252,10 +272,14 @@ def main():
         peaks, peak_src = _load_peaks()
         a_ms = statistics.mean(a_eval_ms)
         a_points = stats["visits"][8]          # L9 points: one launch evaluates all of them
-        ops_per_point = 2                      # one multiply-add forming dim_m_a*dim_n_a, one compare
+        # Roofline: every point needs one product and one
+        # compare = 2 integer ops.  Peak = issue-bound integer lane rate with
+        # 16-bit SIMD (one 32-bit lane instruction carries two 16-bit ops):
+        # SMs x 4 sub-partitions x 32 lanes x 2 halves x sm_max_mhz.
+        ops_per_point = 2
         sm_count = torch.cuda.get_device_properties(0).multi_processor_count
-        lanes = 128                            # int lanes / clk / SM: ALU pipe 64 + FMA pipe 64
-        peak_ops = sm_count * lanes * float(peaks.get("sm_max_mhz", 1965.0)) * 1e6
+        lanes = 128                            # integer lane-instructions / clk / SM (4 x 32, ALU + FMA pipes)
+        peak_ops = sm_count * lanes * 2 * float(peaks.get("sm_max_mhz", 1965.0)) * 1e6
         achieved = ops_per_point * a_points / (a_ms / 1e3) / world if a_ms > 0 else 0.0
         traffic = None
         prof = os.path.join(ROOT, "profiles", "k_eval_traffic.json")
@@ -277,12 +301,13 @@ def main():
                        "l2": "flushed between timed steps (256 MiB write)", "parallelism": "dp%d" % world},
             "survivors_per_s": survivors / (ms / 1e3),
             "roofline": {"bound": "alu", "kernel": "k_eval<A> (L8-L9 A-read grids)",
-                         "achieved": achieved / 1e12, "peak": peak_ops / 1e12, "unit": "Tops/s",
+                         "achieved": achieved / 1e12, "peak": peak_ops / 1e12, "unit": "T int16-ops/s",
                          "frac": achieved / peak_ops if peak_ops else None, "traffic": traffic,
                          "algorithmic_ops_per_launch": ops_per_point * a_points // world,
                          "avg_launch_ms": a_ms,
-                         "peak_source": "%d SMs x %d int lanes/clk x sm_max_mhz (%s MEASURED_PEAKS.json)"
-                                        % (sm_count, lanes, peak_src)},
+                         "peak_source": "%d SMs x %d int lane-instr/clk x 2 (16-bit halves) x sm_max_mhz (%s "
+                                        "MEASURED_PEAKS.json); 2 int ops per point" % (sm_count, lanes, peak_src),
+                         "points_per_s_kernel": a_points / (a_ms / 1e3) if a_ms > 0 else None},
             "e2e": {"value": n_canon / (e2e_step / 1e3), "unit": UNIT,
                     "h2d_bytes_per_step": 96,
                     "d2h_bytes_per_step": 16 * st_local["survivors"] + 512},

@@ -153,57 +153,70 @@ __device__ __forceinline__ uint64_t cta_exclusive_scan64(uint64_t v, uint64_t *s
 // A grid row holds its short-axis coordinate s fixed while the long-axis
 // coordinate j runs 1..L, so the row's points are the products s*j, j <= L.
 //
-// Two points per 32-bit lane: with J = j1 | j2 << 16 (j2 = j1 + 1) and
-// C = (2^16 - T) * 0x10001, the word s*J + C (mod 2^32) holds
-// (s*j1 - T) mod 2^16 in its low half and (s*j2 - T) mod 2^16 in its high half
-// whenever s*j1 < T (no carry reaches the high half) — in particular whenever
-// s*j2 == T.  So a point with s*j == T always leaves a zero half (no false
-// negatives); a zero half can also come from s*j == T (mod 2^16) with
-// s*j != T, which the exact check after the loop rejects.  One IMAD or IADD
-// forms a pair, and ptxas fuses two min.u16x2 into one VIMNMX3.U16x2 that
-// folds two pairs into the row's running minimum: 16 points cost 8 product
-// instructions + 4 min instructions.
-__device__ __forceinline__ uint32_t eval16p(uint32_t acc, uint32_t C, uint32_t s, uint32_t d2) {
+// Each lane evaluates TWO rows s1 < s2 of the same job at once, one per
+// 16-bit half: with Sp = s1 | s2 << 16 and C = (2^16 - T) * 0x10001, the
+// word Sp*j + C (mod 2^32) holds (s1*j - T) mod 2^16 in its low half and
+// (s2*j - T) mod 2^16 in its high half whenever s1*j < T (no carry reaches
+// the high half) — in particular whenever s2*j == T, because s1 < s2.  So a
+// point with s*j == T always leaves a zero half (no false negatives); a zero
+// half can also come from s*j == T (mod 2^16) with s*j != T, which the exact
+// check after the loop rejects.  One IMAD forms a pair of points, and ptxas
+// fuses two min.u16x2 into one VIMNMX3.U16x2 folding two pairs into the
+// running per-half minimum: 32 points cost 16 IMAD + 8 VIMNMX3.
+__device__ __forceinline__ uint32_t eval16pp(uint32_t acc, uint32_t Cb, uint32_t Sp) {
     asm volatile(
-        "{\n\t.reg .b32 t<8>;\n\t"
-        "mad.lo.u32 t0, %2, 0x00020001, %1;\n\t"
-        "add.u32 t1, t0, %3;\n\t"
+        "{\n\t.reg .b32 t<16>;\n\t"
+        "mad.lo.u32 t0, %2, 1, %1;\n\t mad.lo.u32 t1, %2, 2, %1;\n\t"
         "min.u16x2 %0, %0, t0;\n\t min.u16x2 %0, %0, t1;\n\t"
-        "mad.lo.u32 t2, %2, 0x00060005, %1;\n\t"
-        "mad.lo.u32 t3, %2, 0x00080007, %1;\n\t"
+        "mad.lo.u32 t2, %2, 3, %1;\n\t mad.lo.u32 t3, %2, 4, %1;\n\t"
         "min.u16x2 %0, %0, t2;\n\t min.u16x2 %0, %0, t3;\n\t"
-        "mad.lo.u32 t4, %2, 0x000a0009, %1;\n\t"
-        "add.u32 t5, t4, %3;\n\t"
+        "mad.lo.u32 t4, %2, 5, %1;\n\t mad.lo.u32 t5, %2, 6, %1;\n\t"
         "min.u16x2 %0, %0, t4;\n\t min.u16x2 %0, %0, t5;\n\t"
-        "mad.lo.u32 t6, %2, 0x000e000d, %1;\n\t"
-        "mad.lo.u32 t7, %2, 0x0010000f, %1;\n\t"
+        "mad.lo.u32 t6, %2, 7, %1;\n\t mad.lo.u32 t7, %2, 8, %1;\n\t"
         "min.u16x2 %0, %0, t6;\n\t min.u16x2 %0, %0, t7;\n\t"
+        "mad.lo.u32 t8, %2, 9, %1;\n\t mad.lo.u32 t9, %2, 10, %1;\n\t"
+        "min.u16x2 %0, %0, t8;\n\t min.u16x2 %0, %0, t9;\n\t"
+        "mad.lo.u32 t10, %2, 11, %1;\n\t mad.lo.u32 t11, %2, 12, %1;\n\t"
+        "min.u16x2 %0, %0, t10;\n\t min.u16x2 %0, %0, t11;\n\t"
+        "mad.lo.u32 t12, %2, 13, %1;\n\t mad.lo.u32 t13, %2, 14, %1;\n\t"
+        "min.u16x2 %0, %0, t12;\n\t min.u16x2 %0, %0, t13;\n\t"
+        "mad.lo.u32 t14, %2, 15, %1;\n\t mad.lo.u32 t15, %2, 16, %1;\n\t"
+        "min.u16x2 %0, %0, t14;\n\t min.u16x2 %0, %0, t15;\n\t"
         "}"
         : "+r"(acc)
-        : "r"(C), "r"(s), "r"(d2));
+        : "r"(Cb), "r"(Sp));
     return acc;
 }
 
-// Whole row: the points s*1 .. s*L against T (T <= 65535, s, L <= 4095).
-// The loop runs ceil(L/16) blocks; products past L are computed but a match
-// there is rejected by the exact check (j = T/s must satisfy j <= L).
-// Returns the unique j in [1, L] with s*j == T, or 0.  s == 0 marks an idle
-// lane.  T/s is formed with the fp32 reciprocal: for T < 2^16 and s < 2^12
-// its error is far below 1/2, so rounding gives the exact quotient whenever
-// s divides T, and the integer check s*j == T decides.
-__device__ __forceinline__ uint32_t eval_row(uint32_t s, uint32_t T, uint32_t L) {
-    uint32_t C = (0x10000u - T) * 0x10001u;
-    const uint32_t step = s * 0x00100010u;   // +16 on each half's index
-    const uint32_t d2 = s * 0x00020002u;     // +2 on each half's index
-    uint32_t acc = 0xffffffffu;
-    for (uint32_t j = 0; j < L; j += 16) {
-        acc = eval16p(acc, C, s, d2);
-        C += step;
-    }
-    const bool cand = s != 0 && ((acc & 0xffffu) == 0 || (acc >> 16) == 0);
-    if (!cand) return 0;
+// Exact check of one candidate row: returns the unique j in [1, L] with
+// s*j == T, or 0.  T/s is formed with the fp32 reciprocal: for T < 2^16 and
+// s < 2^12 its error is far below 1/2, so rounding gives the exact quotient
+// whenever s divides T, and the integer check s*j == T decides.
+__device__ __forceinline__ uint32_t exact_hit(uint32_t s, uint32_t T, uint32_t L) {
+    if (s == 0) return 0;
     const uint32_t t = __float2uint_rn(__fdividef((float)T, (float)s));
     return (t * s == T && t <= L) ? t : 0u;
+}
+
+// Rows s1 < s2 (s2 == 0: single row) of one job against T over j = 1..L
+// (T <= 65535, s, L <= 4095).  The loop runs ceil(L/16) blocks; products past
+// L are computed but a match there is rejected by the exact check (j <= L).
+// Returns the long coordinates of the two rows' a1/b1 passes (0 = none).
+struct RowPairHits { uint32_t t1, t2; };
+__device__ __forceinline__ RowPairHits eval_rows(uint32_t s1, uint32_t s2, uint32_t T, uint32_t L) {
+    const uint32_t Sp = s1 | (s2 << 16);
+    uint32_t Cb = (0x10000u - T) * 0x10001u;
+    asm volatile("" : "+r"(Cb));             // keep C as one register (no per-block re-derivation)
+    const uint32_t step = Sp << 4;           // Sp * 16: advance both rows by 16 points
+    uint32_t acc = 0xffffffffu;
+    for (uint32_t j = 0; j < L; j += 16) {
+        acc = eval16pp(acc, Cb, Sp);
+        Cb += step;
+    }
+    RowPairHits h{0u, 0u};
+    if ((acc & 0xffffu) == 0) h.t1 = exact_hit(s1, T, L);
+    if ((acc >> 16) == 0) h.t2 = exact_hit(s2, T, L);
+    return h;
 }
 
 }  // namespace beast
