@@ -217,6 +217,19 @@ int beast_enumerate_to_host(beast_space *space, int rank, int world, void *strea
                             beast_record *host_out, uint64_t capacity, uint64_t *written,
                             beast_stats *stats);
 
+/* factorised evaluation (time to solution; NOT the
+ * canonical points/s path): the A and B read-grid sub-nests of a prefix are
+ * independent level sets (§X-B) and cant_reshape_a1/b1
+ * can only be False where dim_m_x * dim_n_x == threads_per_block,
+ * so each prefix's valid A and B grids are found among the divisors of T and
+ * its survivors are their product.  Same survivor count / canonical list as
+ * beast_count / beast_enumerate (checked by the parity tests); no per-point
+ * evaluation and therefore no stats.  Arguments as beast_count /
+ * beast_enumerate. */
+int beast_count_factorized(beast_space *space, int rank, int world, void *stream, uint64_t *survivors);
+int beast_enumerate_factorized(beast_space *space, int rank, int world, void *stream, beast_record *out,
+                               uint64_t capacity, uint64_t *written);
+
 /* Order-sensitive digest of n device records:
  *   sum_i sm64(sm64(hi_i ^ sm64(base + i)) ^ lo_i) mod 2^64,
  * sm64 = splitmix64 finaliser.  Partial digests of consecutive shards (with

@@ -113,6 +113,25 @@ def beast_enumerate_to_host(handle, out, rank=0, world=1, stream=None, stats=Fal
     return (int(n.value), stats_dict(st)) if stats else int(n.value)
 
 
+def beast_count_factorized(handle, rank=0, world=1, stream=None) -> int:
+    """Survivor count by the factorised (divisor) evaluation — time to
+    solution, not a points/s path (SURVEY §8(f) NEXT #1)."""
+    n = ctypes.c_uint64(0)
+    _check(_lib.lib().beast_count_factorized(handle, rank, world, _stream_ptr(stream), ctypes.byref(n)), handle)
+    return int(n.value)
+
+
+def beast_enumerate_factorized(handle, out, rank=0, world=1, stream=None) -> int:
+    n = ctypes.c_uint64(0)
+    cap = out.shape[0] if out is not None else 0
+    ptr = ctypes.c_void_p(out.data_ptr()) if out is not None and cap else None
+    rc = _lib.lib().beast_enumerate_factorized(handle, rank, world, _stream_ptr(stream), ptr, cap, ctypes.byref(n))
+    if rc == BEAST_ERR_CAPACITY:
+        raise BeastError(rc, "need %d records" % n.value)
+    _check(rc, handle)
+    return int(n.value)
+
+
 def beast_digest(records, base=0, stream=None) -> int:
     """Digest of a CUDA uint64 (n, 2) [lo, hi] record tensor."""
     d = ctypes.c_uint64(0)
@@ -192,6 +211,17 @@ class Space:
         r = beast_enumerate(self.handle, out, rank, world, stream, stats)
         n = r[0] if stats else r
         return (out[:n], r[1]) if stats else out[:n]
+
+    def count_factorized(self, rank=0, world=1, stream=None):
+        return beast_count_factorized(self.handle, rank, world, stream)
+
+    def enumerate_factorized(self, rank=0, world=1, stream=None, out=None):
+        import torch
+        if out is None:
+            n = self.count_factorized(rank, world, stream)
+            out = torch.empty((max(n, 1), 2), dtype=torch.uint64, device="cuda")
+        n = beast_enumerate_factorized(self.handle, out, rank, world, stream)
+        return out[:n]
 
     def set_timing(self, enable=True):
         _check(_lib.lib().beast_space_set_timing(self.handle, int(enable)))

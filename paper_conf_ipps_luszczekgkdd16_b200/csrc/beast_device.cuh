@@ -199,17 +199,18 @@ __device__ __forceinline__ uint32_t exact_hit(uint32_t s, uint32_t T, uint32_t L
 }
 
 // Rows s1 < s2 (s2 == 0: single row) of one job against T over j = 1..L
-// (T <= 65535, s, L <= 4095).  The loop runs ceil(L/16) blocks; products past
-// L are computed but a match there is rejected by the exact check (j <= L).
+// (T <= 65535, s, L <= 4095).  The loop runs NB >= ceil(L/16) blocks (NB is
+// uniform across the warp); products past L are computed but a match there is
+// rejected by the exact check (j <= L).
 // Returns the long coordinates of the two rows' a1/b1 passes (0 = none).
 struct RowPairHits { uint32_t t1, t2; };
-__device__ __forceinline__ RowPairHits eval_rows(uint32_t s1, uint32_t s2, uint32_t T, uint32_t L) {
+__device__ __forceinline__ RowPairHits eval_rows(uint32_t s1, uint32_t s2, uint32_t T, uint32_t L, uint32_t NB) {
     const uint32_t Sp = s1 | (s2 << 16);
     uint32_t Cb = (0x10000u - T) * 0x10001u;
     asm volatile("" : "+r"(Cb));             // keep C as one register (no per-block re-derivation)
     const uint32_t step = Sp << 4;           // Sp * 16: advance both rows by 16 points
     uint32_t acc = 0xffffffffu;
-    for (uint32_t j = 0; j < L; j += 16) {
+    for (uint32_t b = 0; b < NB; ++b) {
         acc = eval16pp(acc, Cb, Sp);
         Cb += step;
     }

@@ -209,3 +209,34 @@ def test_limits_from_device_b200(beast):
               "max_shared_mem_per_block", "max_shmem_per_multi_processor"):
         assert getattr(lim, k) == bi.B200_DEVICE[k], (k, getattr(lim, k))
     assert lim.max_blocks_per_multi_processor == 32 and lim.max_registers_per_thread == 255
+
+
+@pytest.mark.parametrize("key", ["tiny_D_00", "tiny_S_01", "tiny_C_10", "tiny_Z_11", "micro_C_00", "k40c_D_00",
+                                 "k40c_S_10", "k40c_C_01", "k40c_Z_11", "b200_D_00", "b200_C_11"])
+def test_factorized_equals_canonical(beast, golden_expected, key):
+    """the divisor-factorised path gives the same count
+    and the same canonical list (digest) as the per-point path / the oracle."""
+    e = golden_expected[key]
+    with beast.Space.from_desc(e["space"]) as sp:
+        assert sp.count_factorized() == e["survivors"]
+        rec = sp.enumerate_factorized()
+        assert len(rec) == e["survivors"]
+        if len(rec):
+            assert "0x%016x" % beast.beast_digest(rec) == e["digest"]
+
+
+@pytest.mark.parametrize("seed", range(0, 200, 7))
+def test_factorized_fuzz(beast, seed):
+    desc = bi.fuzz_space(seed)
+    ref = oracle.nest(desc, records=True)
+    with beast.Space.from_desc(desc) as sp:
+        rec = sp.enumerate_factorized().cpu().numpy()
+    assert np.array_equal(rec, _oracle_lohi(ref["records"]))
+
+
+def test_factorized_shards(beast):
+    desc = bi.headline()
+    with beast.Space.from_desc(desc) as sp:
+        full = sp.enumerate_factorized().cpu().numpy()
+        parts = [sp.enumerate_factorized(rank=r, world=3).cpu().numpy() for r in range(3)]
+    assert np.array_equal(np.concatenate(parts), full)
