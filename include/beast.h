@@ -217,6 +217,22 @@ int beast_enumerate_to_host(beast_space *space, int rank, int world, void *strea
                             beast_record *host_out, uint64_t capacity, uint64_t *written,
                             beast_stats *stats);
 
+/* Stream-ordered enumeration without a host wait.  Enqueues on `stream` the
+ * pass that an earlier synchronous beast_enumerate captured for the same
+ * (rank, world, out, capacity) -- stats off, the handle's current timing
+ * setting -- and returns at once; `out` is complete when the stream reaches
+ * the end of the pass.  Passes on one handle must be issued from one host
+ * thread.  BEAST_ERR_INVALID_ARGUMENT if no such captured pass exists (call
+ * beast_enumerate first). */
+int beast_enumerate_async(beast_space *space, int rank, int world, void *stream,
+                          beast_record *out, uint64_t capacity);
+
+/* Wait for the most recent pass of the handle (synchronous or asynchronous)
+ * to complete; *written: host, out, the records of that pass.
+ * BEAST_ERR_CAPACITY if they exceeded the capacity of the last
+ * beast_enumerate_async. */
+int beast_wait(beast_space *space, void *stream, uint64_t *written);
+
 /* factorised evaluation (time to solution; NOT the
  * canonical points/s path): the A and B read-grid sub-nests of a prefix are
  * independent level sets (§X-B) and cant_reshape_a1/b1

@@ -113,6 +113,24 @@ def beast_enumerate_to_host(handle, out, rank=0, world=1, stream=None, stats=Fal
     return (int(n.value), stats_dict(st)) if stats else int(n.value)
 
 
+def beast_enumerate_async(handle, out, rank=0, world=1, stream=None) -> None:
+    """Enqueue a pass captured by an earlier beast_enumerate with the same
+    (rank, world, out) and return without waiting (see beast_wait)."""
+    cap = out.shape[0] if out is not None else 0
+    ptr = ctypes.c_void_p(out.data_ptr()) if out is not None and cap else None
+    _check(_lib.lib().beast_enumerate_async(handle, rank, world, _stream_ptr(stream), ptr, cap), handle)
+
+
+def beast_wait(handle, stream=None) -> int:
+    """Wait for the handle's most recent pass; returns its record count."""
+    n = ctypes.c_uint64(0)
+    rc = _lib.lib().beast_wait(handle, _stream_ptr(stream), ctypes.byref(n))
+    if rc == BEAST_ERR_CAPACITY:
+        raise BeastError(rc, "need %d records" % n.value)
+    _check(rc, handle)
+    return int(n.value)
+
+
 def beast_count_factorized(handle, rank=0, world=1, stream=None) -> int:
     """Survivor count by the factorised (divisor) evaluation — time to
     solution, not a points/s path (SURVEY §8(f) NEXT #1)."""

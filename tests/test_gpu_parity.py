@@ -240,3 +240,26 @@ def test_factorized_shards(beast):
         full = sp.enumerate_factorized().cpu().numpy()
         parts = [sp.enumerate_factorized(rank=r, world=3).cpu().numpy() for r in range(3)]
     assert np.array_equal(np.concatenate(parts), full)
+
+
+@pytest.mark.gpu
+def test_async_passes_match_sync(beast, golden_expected):
+    """beast_enumerate_async replays the captured pass; several in flight,
+    then beast_wait: same records as the synchronous call."""
+    import torch
+    e = golden_expected["k40c_D_00"]          # the headline space
+    with beast.Space.from_desc(bi.headline()) as sp:
+        out = torch.empty((e["survivors"], 2), dtype=torch.uint64, device="cuda")
+        with pytest.raises(beast.BeastError):
+            beast.beast_enumerate_async(sp.handle, out)          # nothing captured yet
+        n = beast.beast_enumerate(sp.handle, out)
+        ref = out.clone()
+        out.zero_()
+        for _ in range(3):
+            beast.beast_enumerate_async(sp.handle, out)
+        assert beast.beast_wait(sp.handle) == n == e["survivors"]
+        torch.cuda.synchronize()
+        assert torch.equal(out, ref)
+        assert "0x%016x" % beast.beast_digest(out) == e["digest"]
+        # a synchronous call after async ones stays in step
+        assert beast.beast_enumerate(sp.handle, out) == n
