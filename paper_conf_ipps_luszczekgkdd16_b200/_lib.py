@@ -12,7 +12,8 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libbeast.so")
+# BEAST_LIB_PATH (development A/B runs only) selects another in-tree build.
+LIB_PATH = os.environ.get("BEAST_LIB_PATH") or os.path.join(_HERE, "libbeast.so")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(

@@ -162,10 +162,21 @@ __device__ __forceinline__ uint64_t cta_exclusive_scan64(uint64_t v, uint64_t *s
 // half can also come from s*j == T (mod 2^16) with s*j != T, which the exact
 // check after the loop rejects.  One IMAD forms a pair of points, and ptxas
 // fuses two min.u16x2 into one VIMNMX3.U16x2 folding two pairs into the
-// running per-half minimum: 32 points cost 16 IMAD + 8 VIMNMX3.
-__device__ __forceinline__ uint32_t eval16pp(uint32_t acc, uint32_t Cb, uint32_t Sp) {
+// running per-half minimum; the other half of a block uses the packed
+// add-and-min VIADDMNMX.U16x2: 32 points cost 8 IMAD + 4 VIMNMX3 +
+// 8 VIADDMNMX (measured fastest mix, scripts/micro/scan.cu).
+__device__ __forceinline__ void eval16pp(uint32_t &acc, uint32_t &acc2, uint32_t Cb, uint32_t Sp,
+                                         const uint32_t (&M)[8]) {
+    // j = 1..8: IMAD products folded pairwise by VIMNMX3 (FMA-heavy + ALU
+    // pipes); j = 9..16: one packed add-and-min per pair of points,
+    // min(acc, Cb + M[j-9]) per 16-bit half (VIADDMNMX.U16x2, ALU pipe),
+    // with the loop invariants M[i] = (9 + i) * Sp.  The halves of Cb + M
+    // are formed mod 2^16 without a carry between them; the high half of Cb
+    // itself carries no low-half carry whenever the high row has a true
+    // match (see scan_rows), so both forms leave a zero exactly where the
+    // IMAD form does.
     asm volatile(
-        "{\n\t.reg .b32 t<16>;\n\t"
+        "{\n\t.reg .b32 t<8>;\n\t"
         "mad.lo.u32 t0, %2, 1, %1;\n\t mad.lo.u32 t1, %2, 2, %1;\n\t"
         "min.u16x2 %0, %0, t0;\n\t min.u16x2 %0, %0, t1;\n\t"
         "mad.lo.u32 t2, %2, 3, %1;\n\t mad.lo.u32 t3, %2, 4, %1;\n\t"
@@ -174,50 +185,71 @@ __device__ __forceinline__ uint32_t eval16pp(uint32_t acc, uint32_t Cb, uint32_t
         "min.u16x2 %0, %0, t4;\n\t min.u16x2 %0, %0, t5;\n\t"
         "mad.lo.u32 t6, %2, 7, %1;\n\t mad.lo.u32 t7, %2, 8, %1;\n\t"
         "min.u16x2 %0, %0, t6;\n\t min.u16x2 %0, %0, t7;\n\t"
-        "mad.lo.u32 t8, %2, 9, %1;\n\t mad.lo.u32 t9, %2, 10, %1;\n\t"
-        "min.u16x2 %0, %0, t8;\n\t min.u16x2 %0, %0, t9;\n\t"
-        "mad.lo.u32 t10, %2, 11, %1;\n\t mad.lo.u32 t11, %2, 12, %1;\n\t"
-        "min.u16x2 %0, %0, t10;\n\t min.u16x2 %0, %0, t11;\n\t"
-        "mad.lo.u32 t12, %2, 13, %1;\n\t mad.lo.u32 t13, %2, 14, %1;\n\t"
-        "min.u16x2 %0, %0, t12;\n\t min.u16x2 %0, %0, t13;\n\t"
-        "mad.lo.u32 t14, %2, 15, %1;\n\t mad.lo.u32 t15, %2, 16, %1;\n\t"
-        "min.u16x2 %0, %0, t14;\n\t min.u16x2 %0, %0, t15;\n\t"
         "}"
         : "+r"(acc)
         : "r"(Cb), "r"(Sp));
-    return acc;
+#pragma unroll
+    for (int i = 0; i < 8; ++i)
+        asm volatile("{\n\t.reg .b32 t;\n\tadd.u16x2 t, %1, %2;\n\tmin.u16x2 %0, %0, t;\n\t}"
+                     : "+r"(acc2) : "r"(Cb), "r"(M[i]));
 }
 
-// Exact check of one candidate row: returns the unique j in [1, L] with
-// s*j == T, or 0.  T/s is formed with the fp32 reciprocal: for T < 2^16 and
-// s < 2^12 its error is far below 1/2, so rounding gives the exact quotient
-// whenever s divides T, and the integer check s*j == T decides.
-__device__ __forceinline__ uint32_t exact_hit(uint32_t s, uint32_t T, uint32_t L) {
-    if (s == 0) return 0;
-    const uint32_t t = __float2uint_rn(__fdividef((float)T, (float)s));
-    return (t * s == T && t <= L) ? t : 0u;
+__device__ __forceinline__ uint32_t vmin_u16x2(uint32_t a, uint32_t b) {
+    uint32_t r;
+    asm("min.u16x2 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
+    return r;
 }
 
-// Rows s1 < s2 (s2 == 0: single row) of one job against T over j = 1..L
-// (T <= 65535, s, L <= 4095).  The loop runs NB >= ceil(L/16) blocks (NB is
-// uniform across the warp); products past L are computed but a match there is
-// rejected by the exact check (j <= L).
-// Returns the long coordinates of the two rows' a1/b1 passes (0 = none).
-struct RowPairHits { uint32_t t1, t2; };
-__device__ __forceinline__ RowPairHits eval_rows(uint32_t s1, uint32_t s2, uint32_t T, uint32_t L, uint32_t NB) {
+// Zero halves of the packed scan of a row pair: rows s1 < s2 (s2 == 0:
+// single row) of one job against T over j = 1..L (T <= 65535, s, L <= 4095).
+// The loop runs NB >= ceil(L/16) blocks (NB is uniform across the warp);
+// products past L are computed but a match there is rejected by the exact
+// check (t <= L).  Returns the running per-half minimum: a zero half marks a
+// candidate row.
+__device__ __forceinline__ uint32_t scan_rows(uint32_t s1, uint32_t s2, uint32_t T, uint32_t NB) {
     const uint32_t Sp = s1 | (s2 << 16);
     uint32_t Cb = (0x10000u - T) * 0x10001u;
     asm volatile("" : "+r"(Cb));             // keep C as one register (no per-block re-derivation)
     const uint32_t step = Sp << 4;           // Sp * 16: advance both rows by 16 points
-    uint32_t acc = 0xffffffffu;
+    uint32_t M[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) M[i] = Sp * (uint32_t)(9 + i);   // halves exact: 16 * 4095 < 2^16
+    uint32_t acc = 0xffffffffu, acc2 = 0xffffffffu;   // two chains: IMAD/VIMNMX3 and VIADDMNMX
     for (uint32_t b = 0; b < NB; ++b) {
-        acc = eval16pp(acc, Cb, Sp);
+        eval16pp(acc, acc2, Cb, Sp, M);
         Cb += step;
     }
-    RowPairHits h{0u, 0u};
-    if ((acc & 0xffffu) == 0) h.t1 = exact_hit(s1, T, L);
-    if ((acc >> 16) == 0) h.t2 = exact_hit(s2, T, L);
-    return h;
+    return vmin_u16x2(acc, acc2);
+}
+
+// fp32 reciprocal (MUFU.RCP, flush-to-zero: operands are integers >= 1 or 0)
+__device__ __forceinline__ float rcp_ftz(float x) {
+    float r;
+    asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+    return r;
+}
+
+// Exact, branch-free check of one candidate row s (0 = idle half) of a job
+// with threads_per_block T and grid sides S (short) x L (long), after the
+// packed scan left `zero` (the row's half of the running minimum is 0):
+//   *t    = T / s when s * t == T and t <= L (the a1/b1 pass), else garbage
+//   a1    = the scan found the row's zero and s * t == T, t <= L
+//   valid = a1 and the divisibility predicate is False: xdiv, s | S, t | L.
+// Quotients are formed with the fp32 reciprocal: for a < 2^16 and d < 2^16
+// the relative error of a * rcp(d) is ~2^-22, far below 1/2 of the quotient's
+// unit, so rounding gives a / d exactly whenever d divides a, and the integer
+// products decide (a wrong quotient can only fail a product check).
+struct RowCheck { uint32_t t; bool a1, valid; };
+__device__ __forceinline__ RowCheck check_row(uint32_t s, bool zero, uint32_t T, uint32_t S, uint32_t L,
+                                              float fT, float fS, float fL, bool xdiv) {
+    const float r = rcp_ftz((float)s);
+    RowCheck c;
+    c.t = __float2uint_rn(fT * r);
+    const uint32_t q = __float2uint_rn(fS * r);
+    const uint32_t u = __float2uint_rn(fL * rcp_ftz((float)c.t));
+    c.a1 = zero && c.t * s == T && c.t <= L;
+    c.valid = c.a1 && xdiv && q * s == S && u * c.t == L;
+    return c;
 }
 
 }  // namespace beast

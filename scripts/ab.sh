@@ -1,0 +1,15 @@
+#!/bin/bash
+# usage (on the GPU box): scripts/ab.sh WORKLOAD variant.so... — bench line per in-tree library build
+WL=$1; shift
+for v in "" "$@"; do
+  BEAST_LIB_PATH=$v timeout 300 python bench.py --workload $WL --no-cpu-baseline --steps 100 > gpurun_out/ab.json 2> gpurun_out/ab.err
+  python - "${v:-default}" <<'PY'
+import json, sys
+try:
+    d = json.load(open("gpurun_out/ab.json"))
+    print("%-40s" % sys.argv[1], d["config"]["workload"], "ms/step %.4f" % d["ms_per_step"], "frac %.4f" % d["roofline"]["frac"],
+          "keval_ms %.4f" % d["roofline"]["avg_launch_ms"], "stages", ["%.4f" % x for x in d.get("stages_ms", [])])
+except Exception as e:
+    print(sys.argv[1], "FAILED", e, open("gpurun_out/ab.err").read()[-500:])
+PY
+done
