@@ -172,6 +172,7 @@ def main():
     ap.add_argument("--workload", default="headline", choices=sorted(WORKLOADS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-sweep", action="store_true", help="skip the batched-sweep (NEXT #3) measurement")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":
@@ -307,6 +308,10 @@ def main():
                 "note": "time to solution of the same survivor list by divisor factorisation "
                         "(beast_enumerate_factorized); not a points/s figure"}
 
+    sweep = None
+    if world == 1 and not args.no_sweep:
+        sweep = sweep_measure(beast, beast_inputs, stream, flush)
+
     line = None
     if rank == 0:
         peaks, peak_src = _load_peaks()
@@ -359,6 +364,7 @@ def main():
                       "flushed before each step, counts checked after the loop); roofline: k_eval<A> "
                       "launches timed by CUDA events in a second loop of synchronous flushed steps",
             "factorised": fact,
+            "sweep": sweep,
             "paper_context": PAPER_CONTEXT,
         }
         print(json.dumps(line), flush=True)
@@ -367,6 +373,49 @@ def main():
         dist.barrier()
         dist.destroy_process_group()
     return 0
+
+
+def sweep_measure(beast, beast_inputs, stream, flush, reps=3):
+    """the 32 configurations the paper tunes one at a
+    time (4 precisions x 4 transposes x {K40c, B200}) counted by one
+    beast_sweep_count call (passes concurrent on internal streams) against
+    the same 32 counting passes issued one after another; CUDA events on the
+    caller's stream, L2 flushed before each repetition."""
+    import torch
+    descs = [(dev, p, ta, tb) for dev in ("k40c", "b200") for p in beast_inputs.PRECISIONS
+             for ta, tb in beast_inputs.TRANSPOSES]
+    spaces = [beast.Space.from_desc(getattr(beast_inputs, dev)(p, ta, tb)) for dev, p, ta, tb in descs]
+    try:
+        counts, stats = beast.sweep(spaces, stream=stream, stats=True)
+        points = sum(st["points"] for st in stats)
+        beast.sweep(spaces, stream=stream)
+        for sp in spaces:
+            sp.count(stream=stream)
+
+        def timed(fn):
+            ms = []
+            for _ in range(reps):
+                flush.zero_()
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                fn()
+                b.record(stream)
+                torch.cuda.synchronize()
+                ms.append(a.elapsed_time(b))
+            return statistics.median(ms)
+
+        got = []
+        sweep_ms = timed(lambda: got.append(beast.sweep(spaces, stream=stream)))
+        seq_ms = timed(lambda: [sp.count(stream=stream) for sp in spaces])
+        assert all(g == counts for g in got)
+        return {"spaces": len(spaces), "configs": "4 precisions x 4 transposes x {K40c, B200}",
+                "survivors": sum(counts), "points": points, "ms": sweep_ms, "sequential_ms": seq_ms,
+                "points_per_s": points / (sweep_ms / 1e3), "speedup_vs_sequential": seq_ms / sweep_ms,
+                "note": "beast_sweep_count (canonical counting passes, concurrent); each pass evaluates "
+                        "every canonical point of its space"}
+    finally:
+        for sp in spaces:
+            sp.close()
 
 
 def cpu_baseline(desc):

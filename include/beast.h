@@ -233,6 +233,23 @@ int beast_enumerate_async(beast_space *space, int rank, int world, void *stream,
  * beast_enumerate_async. */
 int beast_wait(beast_space *space, void *stream, uint64_t *written);
 
+/* batched sweep: count the survivors of n independent
+ * spaces in one call, e.g. the 4 precisions x 4 transposes x {K40c, B200}
+ * configurations the paper tunes one at a time (Fig 10).
+ * Each space's counting pass (the same kernels as beast_count, rank 0 of
+ * world 1) is launched on one of a pool of internal streams forked from
+ * `stream` and joined back to it, so the spaces' passes run concurrently;
+ * then every handle's counters are read.  spaces: host array of n distinct
+ * handles on the current device.  survivors: host, out, n entries.
+ * stats: host, out, n entries or NULL; non-NULL selects the instrumented
+ * passes, and each entry is then the space's per-level visits and
+ * first-failing-predicate rejections (Figs 11-15) -- the attribution table
+ * of the sweep.  A handle without a captured counting pass first runs one
+ * synchronous beast_count.  Errors: BEAST_ERR_INVALID_ARGUMENT (NULL or
+ * repeated handle, handle on another device), any beast_count error. */
+int beast_sweep_count(beast_space *const *spaces, int n, void *stream, uint64_t *survivors,
+                      beast_stats *stats);
+
 /* factorised evaluation (time to solution; NOT the
  * canonical points/s path): the A and B read-grid sub-nests of a prefix are
  * independent level sets (§X-B) and cant_reshape_a1/b1

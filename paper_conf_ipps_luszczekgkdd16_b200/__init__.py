@@ -159,6 +159,23 @@ def beast_digest(records, base=0, stream=None) -> int:
     return int(d.value)
 
 
+def beast_sweep_count(handles, stream=None, stats=False):
+    """survivor counts (and per-space stats) of a batch
+    of spaces, their counting passes run concurrently (include/beast.h)."""
+    n = len(handles)
+    arr = (ctypes.c_void_p * max(n, 1))(*[h.value if isinstance(h, ctypes.c_void_p) else h for h in handles])
+    cnt = (ctypes.c_uint64 * max(n, 1))()
+    st = (beast_stats * max(n, 1))() if stats else None
+    _check(_lib.lib().beast_sweep_count(arr, n, _stream_ptr(stream), cnt, st))
+    counts = [int(cnt[i]) for i in range(n)]
+    return (counts, [stats_dict(st[i]) for i in range(n)]) if stats else counts
+
+
+def sweep(spaces, stream=None, stats=False):
+    """beast_sweep_count over Space objects."""
+    return beast_sweep_count([sp.handle for sp in spaces], stream=stream, stats=stats)
+
+
 def stats_dict(st: beast_stats) -> dict:
     return dict(visits=[int(x) for x in st.visits], rejected=[int(x) for x in st.rejected],
                 survivors=int(st.survivors), prefixes=int(st.prefixes),

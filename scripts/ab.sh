@@ -2,7 +2,7 @@
 # usage (on the GPU box): scripts/ab.sh WORKLOAD variant.so... — bench line per in-tree library build
 WL=$1; shift
 for v in "" "$@"; do
-  BEAST_LIB_PATH=$v timeout 300 python bench.py --workload $WL --no-cpu-baseline --steps 100 > gpurun_out/ab.json 2> gpurun_out/ab.err
+  BEAST_LIB_PATH=$v timeout 300 python bench.py --workload $WL --no-cpu-baseline --no-sweep --steps 100 > gpurun_out/ab.json 2> gpurun_out/ab.err
   python - "${v:-default}" <<'PY'
 import json, sys
 try:

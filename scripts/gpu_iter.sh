@@ -5,7 +5,7 @@ WLS=${@:-headline}
 mkdir -p gpurun_out
 timeout 900 python -m pytest tests -m gpu -x -q 2>&1 | tail -4
 for WL in $WLS; do
-  timeout 300 python bench.py --workload $WL --no-cpu-baseline --steps 100 > gpurun_out/${TAG}_${WL}.json 2> gpurun_out/${TAG}_${WL}.err
+  timeout 300 python bench.py --workload $WL --no-cpu-baseline --no-sweep --steps 100 > gpurun_out/${TAG}_${WL}.json 2> gpurun_out/${TAG}_${WL}.err
   python - gpurun_out/${TAG}_${WL}.json <<'PY'
 import json, sys
 try:
