@@ -173,6 +173,8 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-sweep", action="store_true", help="skip the batched-sweep (NEXT #3) measurement")
+    ap.add_argument("--gather", default="nccl", choices=["nccl", "fused"],
+                    help="N > 1 survivor gather: NCCL point-to-point (default) or the fused NVLink write-out (NEXT #2)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":
@@ -209,7 +211,11 @@ def main():
     gathered = torch.empty((max(survivors, 1), 2), dtype=torch.uint64, device="cuda") if rank == 0 else None
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")   # > 126 MB L2
 
+    fused = bdist.FusedGather(survivors, group=None) if (world > 1 and args.gather == "fused") else None
+
     def step():
+        if fused is not None:
+            return fused.run(sp, stream)
         n = beast.beast_enumerate(sp.handle, out, rank, world, stream)
         if world > 1:
             bdist.gather_records(out[:n], gathered, world)
@@ -343,7 +349,8 @@ def main():
             "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
             "config": {"workload": args.workload, "description": WORKLOADS[args.workload],
                        "n_canon": n_canon, "survivors": survivors,
-                       "l2": "flushed between timed steps (256 MiB write)", "parallelism": "dp%d" % world},
+                       "l2": "flushed between timed steps (256 MiB write)", "parallelism": "dp%d" % world,
+                       "gather": args.gather if world > 1 else None},
             "survivors_per_s": survivors / (ms / 1e3),
             "roofline": {"bound": "alu", "kernel": "k_eval<A> (L8-L9 A-read grids)",
                          "achieved": achieved / 1e12, "peak": peak_ops / 1e12, "unit": "T int16-ops/s",

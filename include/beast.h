@@ -233,6 +233,35 @@ int beast_enumerate_async(beast_space *space, int rank, int world, void *stream,
  * beast_enumerate_async. */
 int beast_wait(beast_space *space, void *stream, uint64_t *written);
 
+/* fused survivor gather (the writer
+ * stores the shard's records straight into rank 0's buffer at the shard's
+ * global offset, over NVLink, instead of a separate NCCL gather).
+ *
+ * beast_enumerate_stage: run shard (rank, world)'s pass up to its canonical
+ * tuple list (prefix stage, flattener, A and B grids, canonical placement;
+ * no write-out) and store the shard's record count (16 per tuple) into
+ * *d_count, a caller-owned DEVICE u64 (8-byte aligned), on `stream`.
+ * *count: host, out, nullable (the same number).  Synchronous.
+ *
+ * beast_write_at: write-out of the staged shard (the last pass on this
+ * handle must be beast_enumerate_stage with the same rank, world): record i
+ * of the shard is stored at out[base + i], base = d_counts[0] + ... +
+ * d_counts[rank - 1], where d_counts is a DEVICE array of `world` u64
+ * (typically the all-gather of every rank's *d_count, produced on `stream`).
+ * `out` is a DEVICE pointer valid in this process -- rank 0's output buffer
+ * mapped into it (CUDA IPC / symmetric memory over NVLink) or a local buffer;
+ * `capacity` = records it holds (16-byte aligned).  *base_out: host, out,
+ * nullable.  Reads d_counts back (one small stream-synchronous copy), then
+ * enqueues the write-out kernel and returns; the records are complete when
+ * `stream` reaches it.  The concatenation over ranks equals the world-1
+ * list.  Errors: BEAST_ERR_INVALID_ARGUMENT (nothing staged for (rank,
+ * world), d_counts[rank] differs from the staged count), BEAST_ERR_CAPACITY
+ * (base + count > capacity; nothing written). */
+int beast_enumerate_stage(beast_space *space, int rank, int world, void *stream, uint64_t *d_count,
+                          uint64_t *count);
+int beast_write_at(beast_space *space, int rank, int world, void *stream, beast_record *out,
+                   uint64_t capacity, const uint64_t *d_counts, uint64_t *base_out);
+
 /* batched sweep: count the survivors of n independent
  * spaces in one call, e.g. the 4 precisions x 4 transposes x {K40c, B200}
  * configurations the paper tunes one at a time (Fig 10).

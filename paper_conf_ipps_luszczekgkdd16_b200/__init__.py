@@ -159,6 +159,26 @@ def beast_digest(records, base=0, stream=None) -> int:
     return int(d.value)
 
 
+def beast_enumerate_stage(handle, d_count, rank=0, world=1, stream=None) -> int:
+    """NEXT #2, phase 1: stage shard (rank, world); d_count: 1-element
+    int64/uint64 CUDA tensor receiving the shard's record count."""
+    n = ctypes.c_uint64(0)
+    _check(_lib.lib().beast_enumerate_stage(handle, rank, world, _stream_ptr(stream),
+                                            ctypes.c_void_p(d_count.data_ptr()), ctypes.byref(n)), handle)
+    return int(n.value)
+
+
+def beast_write_at(handle, out_ptr, capacity, d_counts, rank=0, world=1, stream=None) -> int:
+    """NEXT #2, phase 2: write the staged shard at its global offset into the
+    device buffer at out_ptr (an int address: a local tensor's data_ptr() or
+    rank 0's buffer mapped into this process) of `capacity` records.
+    d_counts: CUDA tensor of `world` record counts.  Returns the base offset."""
+    base = ctypes.c_uint64(0)
+    _check(_lib.lib().beast_write_at(handle, rank, world, _stream_ptr(stream), ctypes.c_void_p(out_ptr), capacity,
+                                     ctypes.c_void_p(d_counts.data_ptr()), ctypes.byref(base)), handle)
+    return int(base.value)
+
+
 def beast_sweep_count(handles, stream=None, stats=False):
     """survivor counts (and per-space stats) of a batch
     of spaces, their counting passes run concurrently (include/beast.h)."""

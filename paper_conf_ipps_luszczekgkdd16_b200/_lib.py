@@ -88,6 +88,8 @@ _sig = {
     "beast_count_factorized": ([_vp, ctypes.c_int, ctypes.c_int, _vp, _u64p], ctypes.c_int),
     "beast_enumerate_factorized": ([_vp, ctypes.c_int, ctypes.c_int, _vp, _vp, ctypes.c_uint64, _u64p],
                                    ctypes.c_int),
+    "beast_enumerate_stage": ([_vp, ctypes.c_int, ctypes.c_int, _vp, _vp, _u64p], ctypes.c_int),
+    "beast_write_at": ([_vp, ctypes.c_int, ctypes.c_int, _vp, _vp, ctypes.c_uint64, _vp, _u64p], ctypes.c_int),
     "beast_sweep_count": ([_P(_vp), ctypes.c_int, _vp, _u64p, _P(beast_stats)], ctypes.c_int),
     "beast_space_set_timing": ([_vp, ctypes.c_int], ctypes.c_int),
     "beast_last_stage_ms": ([_vp, _P(ctypes.c_float)], ctypes.c_int),

@@ -119,3 +119,51 @@ def enumerate_distributed(space, gather=False, stats=False, stream=None) -> dict
     if stats:
         out["stats"] = combine_stats(st, world)
     return out
+
+
+class FusedGather:
+    """fused survivor gather.
+
+    Instead of enumerating into a local buffer and then gathering with NCCL,
+    every rank stages its shard (beast_enumerate_stage: the pass up to the
+    canonical tuple list, its record count into a device word), the counts
+    are all-gathered (NCCL, 8 bytes per rank), and every rank's write-out
+    kernel stores its records directly into rank 0's buffer at the shard's
+    global offset (beast_write_at), the buffer being symmetric memory mapped
+    into every rank over NVLink.  A symmetric-memory barrier then makes the
+    list complete on rank 0.  With one process (no process group) the buffer
+    is an ordinary local tensor.  `capacity` = records the list may hold
+    (the whole space's survivors)."""
+
+    def __init__(self, capacity: int, device=None, group=None):
+        self.world = dist.get_world_size(group) if dist.is_initialized() else 1
+        self.rank = dist.get_rank(group) if dist.is_initialized() else 0
+        self.device = device or torch.device("cuda", torch.cuda.current_device())
+        self.capacity = max(int(capacity), 1)
+        self.group = group
+        self.hdl = None
+        if self.world > 1:
+            import torch.distributed._symmetric_memory as symm_mem
+            self.buf = symm_mem.empty((self.capacity, 2), dtype=torch.int64, device=self.device)
+            self.hdl = symm_mem.rendezvous(self.buf, group if group is not None else dist.group.WORLD)
+            self.root_ptr = int(self.hdl.buffer_ptrs[0])   # rank 0's buffer, mapped into this process
+        else:
+            self.buf = torch.empty((self.capacity, 2), dtype=torch.int64, device=self.device)
+            self.root_ptr = self.buf.data_ptr()
+        self.d_count = torch.zeros(1, dtype=torch.int64, device=self.device)
+        self.d_counts = torch.zeros(self.world, dtype=torch.int64, device=self.device)
+
+    def run(self, space, stream=None) -> int:
+        """One fused enumeration + gather; returns the global record count.
+        On rank 0, self.buf[:total] then holds the canonical list (int64 view
+        of the (lo, hi) records)."""
+        from . import beast_enumerate_stage, beast_write_at
+        beast_enumerate_stage(space.handle, self.d_count, self.rank, self.world, stream)
+        if self.world > 1:
+            dist.all_gather_into_tensor(self.d_counts, self.d_count, group=self.group)
+        else:
+            self.d_counts.copy_(self.d_count)
+        beast_write_at(space.handle, self.root_ptr, self.capacity, self.d_counts, self.rank, self.world, stream)
+        if self.hdl is not None:
+            self.hdl.barrier()
+        return int(self.d_counts.sum().item())
