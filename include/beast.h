@@ -279,6 +279,64 @@ int beast_write_at(beast_space *space, int rank, int world, void *stream, beast_
 int beast_sweep_count(beast_space *const *spaces, int n, void *stream, uint64_t *survivors,
                       beast_stats *stats);
 
+/* generic space IR.  A space written the way the
+ * BEAST language writes one (§V-VIII): iterators whose
+ * [start, stop) ranges with a step are C int64 expressions of constants and
+ * earlier iterators (values start, start+step, ... while < stop for step > 0,
+ * > stop for step < 0), derived variables (C int64 expressions, listing
+ * order) and constraints (C expressions; nonzero prunes, reading A5).  Every
+ * derived variable and constraint belongs to the deepest iterator it reads
+ * (the level-set rule); constraints of one level are tested in
+ * listing order and the first that holds is the point's rejection.  All
+ * strings are copied; names are C identifiers; an expression may read only
+ * names declared before it (in the level sense).  Arithmetic is C int64 (/
+ * and % truncate; an expression must not divide by zero -- guard it with
+ * || or ?:, e.g. "loads == 0 || fmas / loads < 2"). */
+typedef struct beast_ir beast_ir;   /* opaque, library-owned */
+typedef struct {
+    int32_t n_constants;
+    const char *const *constant_names;
+    const int64_t *constant_values;
+    int32_t n_iterators;                          /* <= 64 */
+    const char *const *iterator_names;
+    const char *const *iterator_start, *const *iterator_stop, *const *iterator_step;
+    int32_t n_derived;
+    const char *const *derived_names;
+    const char *const *derived_exprs;
+    int32_t n_constraints;                        /* <= 64 */
+    const char *const *constraint_names;
+    const char *const *constraint_exprs;
+} beast_ir_desc;
+
+/* Validate, assign levels, generate the CUDA source of the space and compile
+ * it for sm_100a with NVRTC (opened at run time; BEAST_NVRTC may name the
+ * library).  Needs no GPU: the cubin is loaded on the current device by the
+ * first count / enumerate.  On failure *out may still receive a
+ * handle whose beast_ir_last_error explains it (destroy it).  Errors:
+ * BEAST_ERR_INVALID_ARGUMENT (bad name, unknown or later-level name in an
+ * expression, NVRTC compile error), BEAST_ERR_UNSUPPORTED (no NVRTC),
+ * BEAST_ERR_CUDA. */
+int beast_ir_create(const beast_ir_desc *desc, beast_ir **out);
+void beast_ir_destroy(beast_ir *ir);
+const char *beast_ir_last_error(const beast_ir *ir);
+/* The generated CUDA source (owned by the handle). */
+const char *beast_ir_source(const beast_ir *ir);
+/* Level (0-based iterator index, -1 = constants only) of every derived
+ * variable and constraint; host arrays, nullable. */
+int beast_ir_levels(const beast_ir *ir, int32_t *derived_levels, int32_t *constraint_levels);
+/* Count the survivors level by level on `stream` (synchronous).  visits: host,
+ * out, n_iterators loop-body executions per level, nullable; rejected: host,
+ * out, n_constraints first-failing counts, nullable. */
+int beast_ir_count(beast_ir *ir, void *stream, uint64_t *survivors, uint64_t *visits, uint64_t *rejected);
+/* As beast_ir_count, and write the survivors in canonical (lexicographic,
+ * listing-order) order into `out`, a DEVICE buffer of `capacity` rows of
+ * n_iterators int64 values.  *written = survivors.  BEAST_ERR_CAPACITY if
+ * capacity < survivors (nothing of the last level written).  Intermediate
+ * levels are materialised in stream-ordered device allocations
+ * (BEAST_ERR_WORKSPACE if one does not fit). */
+int beast_ir_enumerate(beast_ir *ir, void *stream, int64_t *out, uint64_t capacity, uint64_t *written,
+                       uint64_t *visits, uint64_t *rejected);
+
 /* factorised evaluation (time to solution; NOT the
  * canonical points/s path): the A and B read-grid sub-nests of a prefix are
  * independent level sets (§X-B) and cant_reshape_a1/b1

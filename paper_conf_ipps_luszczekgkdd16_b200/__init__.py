@@ -317,3 +317,95 @@ def unpack(lo: int, hi: int) -> tuple:
     return ((hi >> 52) & m, (hi >> 40) & m, (hi >> 28) & m, (hi >> 16) & m, (hi >> 4) & m,
             (hi >> 1) & 7, hi & 1, (lo >> 52) & m, (lo >> 40) & m, (lo >> 28) & m,
             (lo >> 16) & m, (lo >> 3) & 1, (lo >> 2) & 1, (lo >> 1) & 1, lo & 1)
+
+
+# ----------------------------------------------------------- NEXT #4: generic space IR
+class IRSpace:
+    """A space in the generic IR (include/beast.h beast_ir_desc; the spec dict
+    format of oracle/ir.py: constants, iterators [name, start, stop, step],
+    derived [name, expr], constraints [name, expr]), compiled by the library
+    with NVRTC for sm_100a.  This class only marshals the strings."""
+
+    def __init__(self, spec: dict):
+        import torch  # noqa: F401  (CUDA context on the current device)
+        enc = lambda xs: (ctypes.c_char_p * max(len(xs), 1))(*[x.encode() for x in xs])  # noqa: E731
+        consts = spec.get("constants", {})
+        its = spec["iterators"]
+        der = spec.get("derived", [])
+        con = spec.get("constraints", [])
+        self.names = [i[0] for i in its]
+        self.constraint_names = [c[0] for c in con]
+        self.derived_names = [d[0] for d in der]
+        self._keep = [enc(list(consts)), (ctypes.c_int64 * max(len(consts), 1))(*[int(v) for v in consts.values()]),
+                      enc([i[0] for i in its]), enc([str(i[1]) for i in its]), enc([str(i[2]) for i in its]),
+                      enc([str(i[3]) for i in its]), enc([d[0] for d in der]), enc([d[1] for d in der]),
+                      enc([c[0] for c in con]), enc([c[1] for c in con])]
+        k = self._keep
+        cp = lambda a: ctypes.cast(a, _lib._cpp)  # noqa: E731
+        desc = _lib.beast_ir_desc(len(consts), cp(k[0]), ctypes.cast(k[1], ctypes.POINTER(ctypes.c_int64)),
+                                  len(its), cp(k[2]), cp(k[3]), cp(k[4]), cp(k[5]),
+                                  len(der), cp(k[6]), cp(k[7]), len(con), cp(k[8]), cp(k[9]))
+        h = ctypes.c_void_p()
+        rc = _lib.lib().beast_ir_create(ctypes.byref(desc), ctypes.byref(h))
+        if rc != 0:
+            msg = _lib.lib().beast_ir_last_error(h).decode() if h.value else ""
+            if h.value:
+                _lib.lib().beast_ir_destroy(h)
+            raise BeastError(rc, msg)
+        self.handle = h
+
+    def _err(self, rc):
+        if rc != 0:
+            raise BeastError(rc, _lib.lib().beast_ir_last_error(self.handle).decode())
+
+    @property
+    def source(self) -> str:
+        return _lib.lib().beast_ir_source(self.handle).decode()
+
+    def levels(self) -> dict:
+        d = (ctypes.c_int32 * max(len(self.derived_names), 1))()
+        c = (ctypes.c_int32 * max(len(self.constraint_names), 1))()
+        self._err(_lib.lib().beast_ir_levels(self.handle, d, c))
+        out = {n: i for i, n in enumerate(self.names)}
+        out.update({n: int(d[i]) for i, n in enumerate(self.derived_names)})
+        out.update({n: int(c[i]) for i, n in enumerate(self.constraint_names)})
+        return out
+
+    def count(self, stream=None) -> dict:
+        n = ctypes.c_uint64(0)
+        v = (ctypes.c_uint64 * max(len(self.names), 1))()
+        r = (ctypes.c_uint64 * max(len(self.constraint_names), 1))()
+        self._err(_lib.lib().beast_ir_count(self.handle, _stream_ptr(stream), ctypes.byref(n), v, r))
+        return dict(survivors=int(n.value), visits=[int(x) for x in v[:len(self.names)]],
+                    rejected=[int(x) for x in r[:len(self.constraint_names)]])
+
+    def enumerate(self, stream=None):
+        """Returns (int64 CUDA tensor [survivors, n_iterators], stats dict)."""
+        import torch
+        st = self.count(stream)
+        out = torch.empty((max(st["survivors"], 1), len(self.names)), dtype=torch.int64, device="cuda")
+        n = ctypes.c_uint64(0)
+        v = (ctypes.c_uint64 * max(len(self.names), 1))()
+        r = (ctypes.c_uint64 * max(len(self.constraint_names), 1))()
+        self._err(_lib.lib().beast_ir_enumerate(self.handle, _stream_ptr(stream), ctypes.c_void_p(out.data_ptr()),
+                                               out.shape[0], ctypes.byref(n), v, r))
+        return out[:int(n.value)], dict(survivors=int(n.value), visits=[int(x) for x in v[:len(self.names)]],
+                                         rejected=[int(x) for x in r[:len(self.constraint_names)]])
+
+    def close(self):
+        if getattr(self, "handle", None) is not None and self.handle.value:
+            _lib.lib().beast_ir_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+

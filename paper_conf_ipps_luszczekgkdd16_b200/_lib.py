@@ -58,6 +58,18 @@ class beast_stats(ctypes.Structure):
                 ("valid_a", ctypes.c_uint64), ("tuples", ctypes.c_uint64)]
 
 
+_cpp = ctypes.POINTER(ctypes.c_char_p)
+
+
+class beast_ir_desc(ctypes.Structure):
+    _fields_ = [("n_constants", ctypes.c_int32), ("constant_names", _cpp),
+                ("constant_values", ctypes.POINTER(ctypes.c_int64)),
+                ("n_iterators", ctypes.c_int32), ("iterator_names", _cpp), ("iterator_start", _cpp),
+                ("iterator_stop", _cpp), ("iterator_step", _cpp),
+                ("n_derived", ctypes.c_int32), ("derived_names", _cpp), ("derived_exprs", _cpp),
+                ("n_constraints", ctypes.c_int32), ("constraint_names", _cpp), ("constraint_exprs", _cpp)]
+
+
 ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
 FREE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
 
@@ -91,6 +103,13 @@ _sig = {
     "beast_enumerate_stage": ([_vp, ctypes.c_int, ctypes.c_int, _vp, _vp, _u64p], ctypes.c_int),
     "beast_write_at": ([_vp, ctypes.c_int, ctypes.c_int, _vp, _vp, ctypes.c_uint64, _vp, _u64p], ctypes.c_int),
     "beast_sweep_count": ([_P(_vp), ctypes.c_int, _vp, _u64p, _P(beast_stats)], ctypes.c_int),
+    "beast_ir_create": ([_P(beast_ir_desc), _P(_vp)], ctypes.c_int),
+    "beast_ir_destroy": ([_vp], None),
+    "beast_ir_last_error": ([_vp], ctypes.c_char_p),
+    "beast_ir_source": ([_vp], ctypes.c_char_p),
+    "beast_ir_levels": ([_vp, _P(ctypes.c_int32), _P(ctypes.c_int32)], ctypes.c_int),
+    "beast_ir_count": ([_vp, _vp, _u64p, _u64p, _u64p], ctypes.c_int),
+    "beast_ir_enumerate": ([_vp, _vp, _vp, ctypes.c_uint64, _u64p, _u64p, _u64p], ctypes.c_int),
     "beast_space_set_timing": ([_vp, ctypes.c_int], ctypes.c_int),
     "beast_last_stage_ms": ([_vp, _P(ctypes.c_float)], ctypes.c_int),
     "beast_last_launches": ([_vp, _u64p, _P(ctypes.c_float), _u64p], ctypes.c_int),
