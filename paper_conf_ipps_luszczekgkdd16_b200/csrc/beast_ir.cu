@@ -79,10 +79,8 @@ Nvrtc &nvrtc() {
 }
 
 // ------------------------------------------------------------ the engine
-// Fixed text appended after the generated level functions.  ir_range(k, v)
-// and ir_eval(k, v) read iterator values v[0..k] (v[k] = the candidate value
-// for ir_eval); ir_eval returns 0 (passes level k) or 1 + the index of the
-// first constraint of level k that holds.
+// Fixed helpers placed before the generated per-level kernels (see
+// generate()): trip count of a range, warp sum, the three-phase scan.
 const char *kEngine = R"CUDA(
 typedef unsigned long long u64;
 
@@ -94,76 +92,6 @@ __device__ __forceinline__ u64 ir_trip(i64 lo, i64 hi, i64 st) {
 __device__ __forceinline__ u64 warp_sum(u64 x) {
     for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
     return x;
-}
-
-// Constant-level constraints (no iterator): stats[NI + c] += 1 for the first
-// one that holds; *pruned = 1 + c, or 0.
-extern "C" __global__ void ir_root(u64 *stats, int *pruned) {
-    const int r = ir_eval(-1, nullptr);
-    *pruned = r;
-    if (r) stats[NI + r - 1] += 1;
-}
-
-// One warp per parent tuple (rows of width k): number of children per parent
-// into cnt[p]; visits of level k and first-failing rejections into stats.
-extern "C" __global__ void __launch_bounds__(256) ir_count(int k, const i64 *par, u64 n_par, u64 *cnt, u64 *stats) {
-    const unsigned lane = threadIdx.x & 31;
-    const u64 w0 = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const u64 nw = ((u64)gridDim.x * blockDim.x) >> 5;
-    u64 visits = 0, rej[NC > 0 ? NC : 1];
-    for (int c = 0; c < NC; ++c) rej[c] = 0;
-    i64 v[NI];
-    for (u64 p = w0; p < n_par; p += nw) {
-        for (int j = 0; j < k; ++j) v[j] = par[p * k + j];
-        i64 lo, hi, st;
-        ir_range(k, v, lo, hi, st);
-        const u64 n = st == 0 ? 0ull : ir_trip(lo, hi, st);
-        visits += n;
-        u64 c = 0;
-        for (u64 i = lane; i < n; i += 32) {
-            v[k] = lo + (i64)i * st;
-            const int r = ir_eval(k, v);
-            if (r == 0) ++c;
-            else rej[r - 1] += 1;
-        }
-        c = warp_sum(c);
-        if (lane == 0) cnt[p] = c;
-    }
-    if (lane == 0 && visits) atomicAdd(&stats[k], visits);
-    for (int c = 0; c < NC; ++c) {
-        const u64 x = warp_sum(rej[c]);
-        if (lane == 0 && x) atomicAdd(&stats[NI + c], x);
-    }
-}
-
-// Emission: re-evaluate in order, write child rows (width k + 1) at
-// off[p] + warp rank (canonical order).
-extern "C" __global__ void __launch_bounds__(256) ir_emit(int k, const i64 *par, u64 n_par, const u64 *off, i64 *out) {
-    const unsigned lane = threadIdx.x & 31;
-    const u64 w0 = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const u64 nw = ((u64)gridDim.x * blockDim.x) >> 5;
-    i64 v[NI];
-    for (u64 p = w0; p < n_par; p += nw) {
-        for (int j = 0; j < k; ++j) v[j] = par[p * k + j];
-        i64 lo, hi, st;
-        ir_range(k, v, lo, hi, st);
-        const u64 n = st == 0 ? 0ull : ir_trip(lo, hi, st);
-        u64 pos = off[p];
-        for (u64 base = 0; base < n; base += 32) {
-            const u64 i = base + lane;
-            bool keep = false;
-            if (i < n) {
-                v[k] = lo + (i64)i * st;
-                keep = ir_eval(k, v) == 0;
-            }
-            const unsigned b = __ballot_sync(0xffffffffu, keep);
-            if (keep) {
-                i64 *row = out + (pos + __popc(b & ((1u << lane) - 1u))) * (u64)(k + 1);
-                for (int j = 0; j <= k; ++j) row[j] = v[j];
-            }
-            pos += __popc(b);
-        }
-    }
 }
 
 // Exclusive scan of n counts, three phases (tiles of 2048 = 256 x 8).
@@ -236,7 +164,8 @@ struct beast_ir {
     std::string err;
     int device = -1;
     cudaLibrary_t lib = nullptr;
-    cudaKernel_t k_root = nullptr, k_count = nullptr, k_emit = nullptr, k_tiles = nullptr, k_top = nullptr,
+    std::vector<cudaKernel_t> k_count, k_emit;   // per level
+    cudaKernel_t k_root = nullptr, k_tiles = nullptr, k_top = nullptr,
                  k_add = nullptr;
     int sm_count = 148;
 };
@@ -325,65 +254,135 @@ int analyse(beast_ir *ir) {
     return BEAST_OK;
 }
 
+// Per level k the generated unit holds two kernels, specialised for the
+// level (names bound as C locals, nothing indexed at run time):
+//   ir_count_<k>: one warp per parent tuple (row of k values); binds the
+//     parent's iterators and every derived variable of a shallower level ONCE
+//     per parent, evaluates the range of iterator k, then lane-strided over
+//     its values binds the level's derived variables and tests the level's
+//     constraints in listing order (the first that holds is the rejection);
+//     children per parent -> cnt, visits and rejections -> stats.
+//   ir_emit_<k>: the same evaluation, writing the surviving child rows
+//     (k + 1 values) at off[parent] + warp rank: canonical order.
+// ir_root tests the constant-level constraints once.
 std::string generate(const beast_ir *ir) {
     std::string s;
-    char buf[256];
+    char buf[512];
     s += "// generated by beast_ir_create (SURVEY §8(f) NEXT #4)\n";
     s += "typedef long long i64;\n";
     snprintf(buf, sizeof(buf), "#define NI %d\n#define NC %d\n", ir->ni, ir->nc);
     s += buf;
-    auto consts = [&]() {
-        std::string c;
-        for (size_t i = 0; i < ir->cnames.size(); ++i) {
-            snprintf(buf, sizeof(buf), "    const i64 %s = (i64)(%lldLL); (void)%s;\n", ir->cnames[i].c_str(),
-                     ir->cvals[i], ir->cnames[i].c_str());
-            c += buf;
-        }
-        return c;
-    };
-    // bindings visible at level k: iterators 0..k-1 (k_inclusive: 0..k), and
-    // derived variables of level <= the deepest bound iterator, in order
-    auto bind = [&](int upto) {   // iterators 0..upto bound
-        std::string c;
-        for (int j = 0; j <= upto; ++j) {
-            snprintf(buf, sizeof(buf), "    const i64 %s = ir_v_[%d]; (void)%s;\n", ir->inames[j].c_str(), j,
-                     ir->inames[j].c_str());
-            c += buf;
-        }
-        for (size_t d = 0; d < ir->dnames.size(); ++d)
-            if (ir->dlev[d] <= upto)
-                c += "    const i64 " + ir->dnames[d] + " = (i64)(" + ir->dexpr[d] + "); (void)" + ir->dnames[d] + ";\n";
-        return c;
-    };
-    s += "__device__ __forceinline__ void ir_range(int ir_k_, const i64 *ir_v_, i64 &ir_lo_, i64 &ir_hi_, "
-         "i64 &ir_st_) {\n";
-    s += "    (void)ir_v_;\n";
-    s += "    switch (ir_k_) {\n";
-    for (int k = 0; k < ir->ni; ++k) {
-        snprintf(buf, sizeof(buf), "    case %d: {\n", k);
-        s += buf;
-        s += consts();
-        s += bind(k - 1);
-        s += "    ir_lo_ = (i64)(" + ir->istart[k] + "); ir_hi_ = (i64)(" + ir->istop[k] + "); ir_st_ = (i64)(" +
-             ir->istep[k] + ");\n    return; }\n";
-    }
-    s += "    default: ir_lo_ = ir_hi_ = 0; ir_st_ = 1; return;\n    }\n}\n";
-    s += "__device__ __forceinline__ int ir_eval(int ir_k_, const i64 *ir_v_) {\n";
-    s += "    (void)ir_v_;\n";
-    s += "    switch (ir_k_) {\n";
-    for (int k = -1; k < ir->ni; ++k) {
-        snprintf(buf, sizeof(buf), "    case %d: {\n", k);
-        s += buf;
-        s += consts();
-        s += bind(k);
-        for (size_t c = 0; c < ir->kexpr.size(); ++c)
-            if (ir->klev[c] == k) {
-                s += "    if ((" + ir->kexpr[c] + ")) return " + std::to_string(c + 1) + ";   // " + ir->knames[c] + "\n";
-            }
-        s += "    return 0; }\n";
-    }
-    s += "    default: return 0;\n    }\n}\n";
     s += kEngine;
+    std::string consts;
+    for (size_t i = 0; i < ir->cnames.size(); ++i) {
+        snprintf(buf, sizeof(buf), "    const i64 %s = (i64)(%lldLL); (void)%s;\n", ir->cnames[i].c_str(),
+                 ir->cvals[i], ir->cnames[i].c_str());
+        consts += buf;
+    }
+    auto derived_at = [&](int lo, int hi, const char *ind) {   // derived variables with lo <= level <= hi
+        std::string c;
+        for (size_t d = 0; d < ir->dnames.size(); ++d)
+            if (ir->dlev[d] >= lo && ir->dlev[d] <= hi)
+                c += std::string(ind) + "const i64 " + ir->dnames[d] + " = (i64)(" + ir->dexpr[d] + "); (void)" +
+                     ir->dnames[d] + ";\n";
+        return c;
+    };
+    auto constraints_at = [&](int k, const char *ind, std::vector<int> *idx) {
+        std::string c;
+        int local = 0;
+        for (size_t j = 0; j < ir->kexpr.size(); ++j)
+            if (ir->klev[j] == k) {
+                ++local;
+                c += std::string(ind) + (local == 1 ? "if" : "else if") + " ((" + ir->kexpr[j] + ")) ir_r_ = " +
+                     std::to_string(local) + ";   // " + ir->knames[j] + "\n";
+                if (idx) idx->push_back((int)j);
+            }
+        return c;
+    };
+    // root: constant-level constraints
+    {
+        std::vector<int> idx;
+        s += "extern \"C\" __global__ void ir_root(u64 *ir_stats_, int *ir_pruned_) {\n";
+        s += consts + derived_at(-1, -1, "    ");
+        s += "    int ir_r_ = 0;\n" + constraints_at(-1, "    ", &idx);
+        s += "    int ir_g_ = 0;\n";
+        for (size_t l = 0; l < idx.size(); ++l)
+            s += "    if (ir_r_ == " + std::to_string(l + 1) + ") ir_g_ = " + std::to_string(idx[l] + 1) + ";\n";
+        s += "    *ir_pruned_ = ir_g_;\n    if (ir_g_) ir_stats_[NI + ir_g_ - 1] += 1;\n}\n";
+    }
+    for (int k = 0; k < ir->ni; ++k) {
+        std::vector<int> idx;
+        const std::string cons = constraints_at(k, "            ", &idx);
+        const int nck = (int)idx.size();
+        std::string parent;   // per-parent bindings
+        for (int j = 0; j < k; ++j) {
+            snprintf(buf, sizeof(buf), "        const i64 %s = ir_par_[ir_p_ * %d + %d]; (void)%s;\n",
+                     ir->inames[j].c_str(), k, j, ir->inames[j].c_str());
+            parent += buf;
+        }
+        parent += derived_at(-1, k - 1, "        ");
+        parent += "        const i64 ir_lo_ = (i64)(" + ir->istart[k] + "), ir_hi_ = (i64)(" + ir->istop[k] +
+                  "), ir_st_ = (i64)(" + ir->istep[k] + ");\n";
+        parent += "        const u64 ir_n_ = ir_st_ == 0 ? 0ull : ir_trip(ir_lo_, ir_hi_, ir_st_);\n";
+        std::string point;   // per-value bindings + constraints
+        point += "            const i64 " + ir->inames[k] + " = ir_lo_ + (i64)ir_i_ * ir_st_; (void)" +
+                 ir->inames[k] + ";\n";
+        point += derived_at(k, k, "            ");
+        point += "            int ir_r_ = 0;\n" + cons;
+        const std::string head =
+            "    const unsigned ir_lane_ = threadIdx.x & 31;\n"
+            "    const u64 ir_w0_ = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;\n"
+            "    const u64 ir_nw_ = ((u64)gridDim.x * blockDim.x) >> 5;\n";
+        // count
+        snprintf(buf, sizeof(buf),
+                 "extern \"C\" __global__ void __launch_bounds__(256) ir_count_%d(const i64 *ir_par_, u64 ir_npar_, "
+                 "u64 *ir_cnt_, u64 *ir_stats_) {\n", k);
+        s += buf;
+        s += head + consts;
+        snprintf(buf, sizeof(buf), "    u64 ir_vis_ = 0, ir_rej_[%d];\n    for (int ir_q_ = 0; ir_q_ < %d; ++ir_q_) ir_rej_[ir_q_] = 0;\n",
+                 nck > 0 ? nck : 1, nck);
+        s += buf;
+        s += "    for (u64 ir_p_ = ir_w0_; ir_p_ < ir_npar_; ir_p_ += ir_nw_) {\n" + parent;
+        s += "        ir_vis_ += ir_n_;\n        u64 ir_c_ = 0;\n";
+        s += "        for (u64 ir_i_ = ir_lane_; ir_i_ < ir_n_; ir_i_ += 32) {\n" + point;
+        if (nck) s += "            if (ir_r_ == 0) ++ir_c_; else ir_rej_[ir_r_ - 1] += 1;\n";
+        else s += "            ++ir_c_;\n";
+        s += "        }\n        ir_c_ = warp_sum(ir_c_);\n        if (ir_lane_ == 0) ir_cnt_[ir_p_] = ir_c_;\n    }\n";
+        snprintf(buf, sizeof(buf), "    if (ir_lane_ == 0 && ir_vis_) atomicAdd(&ir_stats_[%d], ir_vis_);\n", k);
+        s += buf;
+        for (int l = 0; l < nck; ++l) {
+            snprintf(buf, sizeof(buf),
+                     "    { const u64 ir_x_ = warp_sum(ir_rej_[%d]); if (ir_lane_ == 0 && ir_x_) atomicAdd(&ir_stats_[NI + %d], ir_x_); }\n",
+                     l, idx[l]);
+            s += buf;
+        }
+        s += "}\n";
+        // emit
+        snprintf(buf, sizeof(buf),
+                 "extern \"C\" __global__ void __launch_bounds__(256) ir_emit_%d(const i64 *ir_par_, u64 ir_npar_, "
+                 "const u64 *ir_off_, i64 *ir_out_) {\n", k);
+        s += buf;
+        s += head + consts;
+        s += "    for (u64 ir_p_ = ir_w0_; ir_p_ < ir_npar_; ir_p_ += ir_nw_) {\n" + parent;
+        s += "        u64 ir_pos_ = ir_off_[ir_p_];\n";
+        s += "        for (u64 ir_b_ = 0; ir_b_ < ir_n_; ir_b_ += 32) {\n";
+        s += "            const u64 ir_i_ = ir_b_ + ir_lane_;\n            bool ir_keep_ = false;\n";
+        s += "            if (ir_i_ < ir_n_) {\n" + point + "            ir_keep_ = ir_r_ == 0;\n            }\n";
+        // the row: the parent's values + this level's value
+        s += "            const unsigned ir_bal_ = __ballot_sync(0xffffffffu, ir_keep_);\n";
+        s += "            if (ir_keep_) {\n";
+        snprintf(buf, sizeof(buf),
+                 "                i64 *ir_row_ = ir_out_ + (ir_pos_ + __popc(ir_bal_ & ((1u << ir_lane_) - 1u))) * %du;\n",
+                 k + 1);
+        s += buf;
+        for (int j = 0; j < k; ++j) {
+            snprintf(buf, sizeof(buf), "                ir_row_[%d] = ir_par_[ir_p_ * %d + %d];\n", j, k, j);
+            s += buf;
+        }
+        snprintf(buf, sizeof(buf), "                ir_row_[%d] = ir_lo_ + (i64)ir_i_ * ir_st_;\n", k);
+        s += buf;
+        s += "            }\n            ir_pos_ += __popc(ir_bal_);\n        }\n    }\n}\n";
+    }
     return s;
 }
 
@@ -423,8 +422,12 @@ int load(beast_ir *ir) {
     IRCK(cudaDeviceGetAttribute(&ir->sm_count, cudaDevAttrMultiProcessorCount, ir->device));
     IRCK(cudaLibraryLoadData(&ir->lib, ir->cubin.data(), nullptr, nullptr, 0, nullptr, nullptr, 0));
     IRCK(cudaLibraryGetKernel(&ir->k_root, ir->lib, "ir_root"));
-    IRCK(cudaLibraryGetKernel(&ir->k_count, ir->lib, "ir_count"));
-    IRCK(cudaLibraryGetKernel(&ir->k_emit, ir->lib, "ir_emit"));
+    ir->k_count.assign(ir->ni, nullptr);
+    ir->k_emit.assign(ir->ni, nullptr);
+    for (int k = 0; k < ir->ni; ++k) {
+        IRCK(cudaLibraryGetKernel(&ir->k_count[k], ir->lib, ("ir_count_" + std::to_string(k)).c_str()));
+        IRCK(cudaLibraryGetKernel(&ir->k_emit[k], ir->lib, ("ir_emit_" + std::to_string(k)).c_str()));
+    }
     IRCK(cudaLibraryGetKernel(&ir->k_tiles, ir->lib, "ir_scan_tiles"));
     IRCK(cudaLibraryGetKernel(&ir->k_top, ir->lib, "ir_scan_top"));
     IRCK(cudaLibraryGetKernel(&ir->k_add, ir->lib, "ir_scan_add"));
@@ -497,8 +500,8 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
         IRCK(cudaMallocAsync((void **)&off, (n_par + 1) * 8, st));
         {
             const long long *pc = par;
-            void *a[] = {(void *)&k, (void *)&pc, (void *)&n_par, (void *)&cnt, (void *)&stats};
-            rc = launch(ir, ir->k_count, grid, 256, st, a);
+            void *a[] = {(void *)&pc, (void *)&n_par, (void *)&cnt, (void *)&stats};
+            rc = launch(ir, ir->k_count[k], grid, 256, st, a);
         }
         if (rc == BEAST_OK) rc = scan(ir, cnt, n_par, off, st, &total);
         long long *child = nullptr;
@@ -517,8 +520,8 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
             }
             if (rc == BEAST_OK) {
                 const long long *pc = par;
-                void *a[] = {(void *)&k, (void *)&pc, (void *)&n_par, (void *)&off, (void *)&child};
-                rc = launch(ir, ir->k_emit, grid, 256, st, a);
+                void *a[] = {(void *)&pc, (void *)&n_par, (void *)&off, (void *)&child};
+                rc = launch(ir, ir->k_emit[k], grid, 256, st, a);
             }
         }
         cudaFreeAsync(cnt, st);
