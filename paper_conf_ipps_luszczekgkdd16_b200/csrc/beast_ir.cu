@@ -111,11 +111,32 @@ extern "C" __global__ void __launch_bounds__(256) ir_scan_tiles(const u64 *in, u
     for (int i = 0; i < 8; ++i) { if (t0 + i < n) out[t0 + i] = run; run += x[i]; }
     if (threadIdx.x == 255) tile_sum[blockIdx.x] = wb + inc;
 }
-extern "C" __global__ void ir_scan_top(u64 *tile_sum, u64 n_tiles, u64 *total) {
-    if (threadIdx.x != 0) return;
-    u64 run = 0;
-    for (u64 t = 0; t < n_tiles; ++t) { const u64 x = tile_sum[t]; tile_sum[t] = run; run += x; }
-    *total = run;
+extern "C" __global__ void __launch_bounds__(1024) ir_scan_top(u64 *tile_sum, u64 n_tiles, u64 *total) {
+    __shared__ u64 s_w[32];
+    __shared__ u64 s_carry;
+    const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    if (threadIdx.x == 0) s_carry = 0;
+    __syncthreads();
+    for (u64 b = 0; b < n_tiles; b += 1024) {
+        const u64 i = b + threadIdx.x;
+        const u64 x = i < n_tiles ? tile_sum[i] : 0ull;
+        u64 inc = x;
+        for (int o = 1; o < 32; o <<= 1) { const u64 y = __shfl_up_sync(0xffffffffu, inc, o); if ((int)lane >= o) inc += y; }
+        if (lane == 31) s_w[warp] = inc;
+        __syncthreads();
+        if (warp == 0) {
+            u64 w = s_w[lane];
+            for (int o = 1; o < 32; o <<= 1) { const u64 y = __shfl_up_sync(0xffffffffu, w, o); if ((int)lane >= o) w += y; }
+            s_w[lane] = w;
+        }
+        __syncthreads();
+        const u64 carry = s_carry;
+        if (i < n_tiles) tile_sum[i] = carry + (warp ? s_w[warp - 1] : 0ull) + inc - x;
+        __syncthreads();
+        if (threadIdx.x == 0) s_carry = carry + s_w[31];
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) *total = s_carry;
 }
 extern "C" __global__ void __launch_bounds__(256) ir_scan_add(u64 *out, u64 n, const u64 *tile_sum, const u64 *total) {
     const u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
@@ -421,6 +442,15 @@ int load(beast_ir *ir) {
     IRCK(cudaGetDevice(&ir->device));
     IRCK(cudaDeviceGetAttribute(&ir->sm_count, cudaDevAttrMultiProcessorCount, ir->device));
     IRCK(cudaLibraryLoadData(&ir->lib, ir->cubin.data(), nullptr, nullptr, 0, nullptr, nullptr, 0));
+    {
+        // the level buffers are stream-ordered allocations from the device's
+        // default pool: keep them mapped between runs (the default release
+        // threshold of 0 would unmap and re-map gigabytes on every call)
+        cudaMemPool_t pool;
+        IRCK(cudaDeviceGetDefaultMemPool(&pool, ir->device));
+        unsigned long long keep = ~0ull;
+        IRCK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep));
+    }
     IRCK(cudaLibraryGetKernel(&ir->k_root, ir->lib, "ir_root"));
     ir->k_count.assign(ir->ni, nullptr);
     ir->k_emit.assign(ir->ni, nullptr);
@@ -453,7 +483,7 @@ int scan(beast_ir *ir, const unsigned long long *cnt, unsigned long long n, unsi
     {
         unsigned long long nt = tiles;
         void *a[] = {(void *)&ts, (void *)&nt, (void *)&tot};
-        if (launch(ir, ir->k_top, 1, 32, st, a) != BEAST_OK) return BEAST_ERR_CUDA;
+        if (launch(ir, ir->k_top, 1, 1024, st, a) != BEAST_OK) return BEAST_ERR_CUDA;
     }
     {
         const unsigned g = (unsigned)std::max(1ull, (n + 255) / 256);
