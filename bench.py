@@ -173,6 +173,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-sweep", action="store_true", help="skip the batched-sweep (NEXT #3) measurement")
+    ap.add_argument("--no-ir", action="store_true", help="skip the generic-IR (NEXT #4) measurement")
     ap.add_argument("--gather", default="nccl", choices=["nccl", "fused"],
                     help="N > 1 survivor gather: NCCL point-to-point (default) or the fused NVLink write-out (NEXT #2)")
     args = ap.parse_args()
@@ -317,6 +318,9 @@ def main():
     sweep = None
     if world == 1 and not args.no_sweep:
         sweep = sweep_measure(beast, beast_inputs, stream, flush)
+    generic_ir = None
+    if world == 1 and not args.no_ir:
+        generic_ir = ir_measure(beast, desc, stream, flush, ms)
 
     line = None
     if rank == 0:
@@ -372,6 +376,7 @@ def main():
                       "launches timed by CUDA events in a second loop of synchronous flushed steps",
             "factorised": fact,
             "sweep": sweep,
+            "generic_ir": generic_ir,
             "paper_context": PAPER_CONTEXT,
         }
         print(json.dumps(line), flush=True)
@@ -423,6 +428,46 @@ def sweep_measure(beast, beast_inputs, stream, flush, reps=3):
     finally:
         for sp in spaces:
             sp.close()
+
+
+def ir_measure(beast, desc, stream, flush, canonical_ms, reps=3):
+    """the same workload written in the generic space IR
+    (tests/ir_specs.gemm_spec: Figs 11-15 as iterators, derived variables and
+    constraints), compiled by the library with NVRTC and counted by the
+    level-wise IR engine; CUDA events on the caller's stream.  The IR spec's
+    constants come from the library's own resolution of the space
+    (beast_space_resolved), not from the oracle."""
+    import torch
+    sys.path.insert(0, os.path.join(ROOT, "tests"))
+    import ir_specs
+    with beast.Space.from_desc(desc) as sp:
+        res = sp.resolved()
+    spec = ir_specs.gemm_spec(res, desc["precision"])
+    t = time.perf_counter()
+    try:
+        ir = beast.IRSpace(spec)
+    except Exception as e:          # no NVRTC on this box: report, do not fail the bench
+        return {"error": str(e)[:200]}
+    compile_s = time.perf_counter() - t
+    with ir:
+        try:
+            st = ir.count(stream=stream)
+        except Exception as e:
+            return {"error": str(e)[:200]}
+        ms = []
+        for _ in range(reps):
+            flush.zero_()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            ir.count(stream=stream)
+            b.record(stream)
+            torch.cuda.synchronize()
+            ms.append(a.elapsed_time(b))
+    m = statistics.median(ms)
+    pts = sum(st["visits"])
+    return {"ms": m, "points": pts, "points_per_s": pts / (m / 1e3), "survivors": st["survivors"],
+            "compile_s": compile_s, "vs_specialised": m / canonical_ms,
+            "note": "generic IR engine (NVRTC-compiled, level-wise) on the same space; counting pass"}
 
 
 def cpu_baseline(desc):
