@@ -163,33 +163,41 @@ __device__ __forceinline__ uint64_t cta_exclusive_scan64(uint64_t v, uint64_t *s
 // check after the loop rejects.  One IMAD forms a pair of points, and ptxas
 // fuses two min.u16x2 into one VIMNMX3.U16x2 folding two pairs into the
 // running per-half minimum; the other half of a block uses the packed
-// add-and-min VIADDMNMX.U16x2: 32 points cost 8 IMAD + 4 VIMNMX3 +
-// 8 VIADDMNMX (measured fastest mix, scripts/micro/scan.cu).
+// add-and-min VIADDMNMX.U16x2.  With KI of the 16 pairs on the IMAD path,
+// 32 points cost KI IMAD (FMA-heavy pipe) + KI/2 VIMNMX3 + (16 - KI)
+// VIADDMNMX (ALU pipe).  In isolation KI = 8 is fastest
+// (scripts/micro/scan.cu), but the rest of k_eval is ALU-heavy (ncu r01e:
+// ALU 66% vs FMA 27% of peak), so the kernel is fastest at KI = 12 (A/B on
+// the B200, headline and SGEMM-B200); the block loop is unrolled twice (the
+// default 16/8/4/1 cascade costs more than it saves at ~5 blocks per row).
+#ifndef BEAST_SCAN_KI
+#define BEAST_SCAN_KI 12
+#endif
+#ifndef BEAST_SCAN_UNROLL
+#define BEAST_SCAN_UNROLL 2
+#endif
+#define BEAST_PRAGMA(x) _Pragma(#x)
+#define BEAST_UNROLL(n) BEAST_PRAGMA(unroll n)
+template <int KI>
 __device__ __forceinline__ void eval16pp(uint32_t &acc, uint32_t &acc2, uint32_t Cb, uint32_t Sp,
-                                         const uint32_t (&M)[8]) {
-    // j = 1..8: IMAD products folded pairwise by VIMNMX3 (FMA-heavy + ALU
-    // pipes); j = 9..16: one packed add-and-min per pair of points,
-    // min(acc, Cb + M[j-9]) per 16-bit half (VIADDMNMX.U16x2, ALU pipe),
-    // with the loop invariants M[i] = (9 + i) * Sp.  The halves of Cb + M
+                                         const uint32_t (&M)[16 - KI + (KI == 16)]) {
+    // j = 1..KI: IMAD products folded pairwise by VIMNMX3 (FMA-heavy + ALU
+    // pipes); j = KI+1..16: one packed add-and-min per pair of points,
+    // min(acc, Cb + M[j-KI-1]) per 16-bit half (VIADDMNMX.U16x2, ALU pipe),
+    // with the loop invariants M[i] = (KI + 1 + i) * Sp.  The halves of Cb + M
     // are formed mod 2^16 without a carry between them; the high half of Cb
     // itself carries no low-half carry whenever the high row has a true
     // match (see scan_rows), so both forms leave a zero exactly where the
     // IMAD form does.
-    asm volatile(
-        "{\n\t.reg .b32 t<8>;\n\t"
-        "mad.lo.u32 t0, %2, 1, %1;\n\t mad.lo.u32 t1, %2, 2, %1;\n\t"
-        "min.u16x2 %0, %0, t0;\n\t min.u16x2 %0, %0, t1;\n\t"
-        "mad.lo.u32 t2, %2, 3, %1;\n\t mad.lo.u32 t3, %2, 4, %1;\n\t"
-        "min.u16x2 %0, %0, t2;\n\t min.u16x2 %0, %0, t3;\n\t"
-        "mad.lo.u32 t4, %2, 5, %1;\n\t mad.lo.u32 t5, %2, 6, %1;\n\t"
-        "min.u16x2 %0, %0, t4;\n\t min.u16x2 %0, %0, t5;\n\t"
-        "mad.lo.u32 t6, %2, 7, %1;\n\t mad.lo.u32 t7, %2, 8, %1;\n\t"
-        "min.u16x2 %0, %0, t6;\n\t min.u16x2 %0, %0, t7;\n\t"
-        "}"
-        : "+r"(acc)
-        : "r"(Cb), "r"(Sp));
 #pragma unroll
-    for (int i = 0; i < 8; ++i)
+    for (int j = 1; j <= KI; j += 2)
+        asm volatile("{\n\t.reg .b32 t0, t1;\n\t"
+                     "mad.lo.u32 t0, %2, %3, %1;\n\t mad.lo.u32 t1, %2, %4, %1;\n\t"
+                     "min.u16x2 %0, %0, t0;\n\t min.u16x2 %0, %0, t1;\n\t}"
+                     : "+r"(acc)
+                     : "r"(Cb), "r"(Sp), "r"((uint32_t)j), "r"((uint32_t)(j + 1)));
+#pragma unroll
+    for (int i = 0; i < 16 - KI; ++i)
         asm volatile("{\n\t.reg .b32 t;\n\tadd.u16x2 t, %1, %2;\n\tmin.u16x2 %0, %0, t;\n\t}"
                      : "+r"(acc2) : "r"(Cb), "r"(M[i]));
 }
@@ -211,12 +219,14 @@ __device__ __forceinline__ uint32_t scan_rows(uint32_t s1, uint32_t s2, uint32_t
     uint32_t Cb = (0x10000u - T) * 0x10001u;
     asm volatile("" : "+r"(Cb));             // keep C as one register (no per-block re-derivation)
     const uint32_t step = Sp << 4;           // Sp * 16: advance both rows by 16 points
-    uint32_t M[8];
+    constexpr int KI = BEAST_SCAN_KI;
+    uint32_t M[16 - KI + (KI == 16)];
 #pragma unroll
-    for (int i = 0; i < 8; ++i) M[i] = Sp * (uint32_t)(9 + i);   // halves exact: 16 * 4095 < 2^16
+    for (int i = 0; i < 16 - KI; ++i) M[i] = Sp * (uint32_t)(KI + 1 + i);   // halves exact: 16 * 4095 < 2^16
     uint32_t acc = 0xffffffffu, acc2 = 0xffffffffu;   // two chains: IMAD/VIMNMX3 and VIADDMNMX
+    BEAST_UNROLL(BEAST_SCAN_UNROLL)
     for (uint32_t b = 0; b < NB; ++b) {
-        eval16pp(acc, acc2, Cb, Sp, M);
+        eval16pp<KI>(acc, acc2, Cb, Sp, M);
         Cb += step;
     }
     return vmin_u16x2(acc, acc2);
