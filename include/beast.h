@@ -227,10 +227,28 @@ int beast_enumerate_to_host(beast_space *space, int rank, int world, void *strea
 int beast_enumerate_async(beast_space *space, int rank, int world, void *stream,
                           beast_record *out, uint64_t capacity);
 
+/* Host-buffer enumeration without a host wait, for pipelining passes of
+ * several handles against their device -> host copies (the copy engine moves
+ * one list over PCIe while the SMs compute the next).  Enqueues on `stream`
+ * the pass that the last successful beast_enumerate_to_host of this handle
+ * captured for (rank, world) -- same device staging buffer, stats off --
+ * followed by the copy of its records into `host_out` (HOST memory of
+ * `capacity` records; pinned, or the copy is not asynchronous), and returns
+ * at once.  The copy length is that earlier call's record count: a handle's
+ * space is fixed, so every pass of one (rank, world) yields the same list;
+ * beast_wait checks it.  `host_out` is valid after beast_wait returns
+ * BEAST_OK.  Errors: BEAST_ERR_INVALID_ARGUMENT if there was no such earlier
+ * call, BEAST_ERR_CAPACITY if its count exceeds `capacity` (nothing is
+ * enqueued). */
+int beast_enumerate_to_host_async(beast_space *space, int rank, int world, void *stream,
+                                  beast_record *host_out, uint64_t capacity);
+
 /* Wait for the most recent pass of the handle (synchronous or asynchronous)
- * to complete; *written: host, out, the records of that pass.
- * BEAST_ERR_CAPACITY if they exceeded the capacity of the last
- * beast_enumerate_async. */
+ * to complete -- and, after beast_enumerate_to_host_async, its host copy;
+ * *written: host, out, the records of that pass.  BEAST_ERR_CAPACITY if they
+ * exceeded the capacity of the last asynchronous call; BEAST_ERR_WORKSPACE if
+ * an asynchronous pass overflowed its scratch or a host pass's count differed
+ * from the copied one. */
 int beast_wait(beast_space *space, void *stream, uint64_t *written);
 
 /* fused survivor gather (the writer

@@ -121,6 +121,15 @@ def beast_enumerate_async(handle, out, rank=0, world=1, stream=None) -> None:
     _check(_lib.lib().beast_enumerate_async(handle, rank, world, _stream_ptr(stream), ptr, cap), handle)
 
 
+def beast_enumerate_to_host_async(handle, out, rank=0, world=1, stream=None) -> None:
+    """Enqueue the pass captured by the handle's last beast_enumerate_to_host
+    for (rank, world) plus the copy of its records into `out` (pinned CPU
+    torch.uint64 tensor (capacity, 2)); returns at once (see beast_wait)."""
+    cap = out.shape[0] if out is not None else 0
+    ptr = ctypes.c_void_p(out.data_ptr()) if out is not None and cap else None
+    _check(_lib.lib().beast_enumerate_to_host_async(handle, rank, world, _stream_ptr(stream), ptr, cap), handle)
+
+
 def beast_wait(handle, stream=None) -> int:
     """Wait for the handle's most recent pass; returns its record count."""
     n = ctypes.c_uint64(0)

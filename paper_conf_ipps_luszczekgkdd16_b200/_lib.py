@@ -97,6 +97,7 @@ _sig = {
     "beast_digest": ([_vp, ctypes.c_uint64, ctypes.c_uint64, _vp, _u64p], ctypes.c_int),
     "beast_enumerate_async": ([_vp, ctypes.c_int, ctypes.c_int, _vp, _vp, ctypes.c_uint64], ctypes.c_int),
     "beast_wait": ([_vp, _vp, _u64p], ctypes.c_int),
+    "beast_enumerate_to_host_async": ([_vp, ctypes.c_int, ctypes.c_int, _vp, _vp, ctypes.c_uint64], ctypes.c_int),
     "beast_count_factorized": ([_vp, ctypes.c_int, ctypes.c_int, _vp, _u64p], ctypes.c_int),
     "beast_enumerate_factorized": ([_vp, ctypes.c_int, ctypes.c_int, _vp, _vp, ctypes.c_uint64, _u64p],
                                    ctypes.c_int),

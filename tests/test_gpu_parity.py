@@ -263,3 +263,39 @@ def test_async_passes_match_sync(beast, golden_expected):
         assert "0x%016x" % beast.beast_digest(out) == e["digest"]
         # a synchronous call after async ones stays in step
         assert beast.beast_enumerate(sp.handle, out) == n
+
+
+@pytest.mark.gpu
+def test_host_async_pipelined_handles(beast, golden_expected):
+    """beast_enumerate_to_host_async on two handles, alternating (pass of one
+    overlapping the other's host copy): every host list equals the golden
+    digest; errors before a synchronous host call and on short capacity."""
+    import torch
+    e = golden_expected["k40c_D_00"]          # the headline space
+    n = e["survivors"]
+    sps = [beast.Space.from_desc(bi.headline()) for _ in range(2)]
+    try:
+        hosts = [torch.empty((n, 2), dtype=torch.uint64).pin_memory() for _ in range(2)]
+        streams = [torch.cuda.Stream() for _ in range(2)]
+        with pytest.raises(beast.BeastError):
+            beast.beast_enumerate_to_host_async(sps[0].handle, hosts[0], stream=streams[0])
+        for sp, h, st in zip(sps, hosts, streams):
+            assert beast.beast_enumerate_to_host(sp.handle, h, stream=st) == n
+        with pytest.raises(beast.BeastError):
+            beast.beast_enumerate_to_host_async(sps[0].handle, hosts[0][: n - 1], stream=streams[0])
+        with pytest.raises(beast.BeastError):
+            beast.beast_enumerate_to_host_async(sps[0].handle, hosts[0], rank=0, world=2, stream=streams[0])
+        for i in range(6):
+            k = i % 2
+            if i >= 2:
+                assert beast.beast_wait(sps[k].handle, streams[k]) == n
+                dev = hosts[k].cuda()
+                assert "0x%016x" % beast.beast_digest(dev) == e["digest"]
+            hosts[k].zero_()
+            beast.beast_enumerate_to_host_async(sps[k].handle, hosts[k], stream=streams[k])
+        for k in range(2):
+            assert beast.beast_wait(sps[k].handle, streams[k]) == n
+            assert "0x%016x" % beast.beast_digest(hosts[k].cuda()) == e["digest"]
+    finally:
+        for sp in sps:
+            sp.close()
