@@ -267,11 +267,12 @@ def main():
     # events on the launching stream, over K synchronous flushed steps.
     sp.set_timing(True)
     step()
-    a_eval_ms = []
+    a_eval_ms, write_ms = [], []
     for i in range(args.steps):
         flush.zero_()
         step()
         a_eval_ms.append(sp.last_launches()[1])
+        write_ms.append(sp.last_write_ms())
     stages = sp.last_stage_ms()
     sp.set_timing(False)
 
@@ -372,6 +373,17 @@ def main():
     if rank == 0:
         peaks, peak_src = _load_peaks()
         a_ms = statistics.mean(a_eval_ms)
+        # survivor write-out (SURVEY §8(d) iii): 16 B per record written by
+        # k_write, against the HBM copy bandwidth of MEASURED_PEAKS.json
+        w_ms = statistics.mean(write_ms) if write_ms and min(write_ms) > 0 else None
+        w_bytes = 16 * st_local["survivors"]
+        write_out = None
+        if w_ms:
+            w_gbs = w_bytes / (w_ms * 1e6)
+            write_out = {"kernel": "k_write", "bytes_per_launch": w_bytes, "avg_launch_ms": w_ms,
+                         "achieved_GBps": w_gbs, "peak_GBps": peaks["hbm_gbs"], "frac": w_gbs / peaks["hbm_gbs"],
+                         "peak_source": "MEASURED_PEAKS.json hbm_gbs (%s; a read+write copy rate, the "
+                                        "write-only kernel is compared against it)" % peak_src}
         a_points = stats["visits"][8]          # L9 points: one launch evaluates all of them
         # Roofline: every point needs one product and one
         # compare = 2 integer ops.  Peak = issue-bound integer lane rate with
@@ -421,6 +433,7 @@ def main():
                            "one step's copy overlaps the next step's pass; host wall clock over %d steps" % n_pipe,
                     "unpipelined": {"value": n_canon / (e2e_sync_step / 1e3), "ms_per_step": e2e_sync_step,
                                     "how": "beast_enumerate_to_host (synchronous), median step"}},
+            "write_out": write_out,
             "gpu_launches": launches,
             "clocks": clk,
             "cpu_baseline": cpu,

@@ -389,6 +389,13 @@ int beast_last_stage_ms(const beast_space *space, float ms[5]);
 int beast_last_launches(const beast_space *space, uint64_t *kernels, float *a_eval_ms,
                         uint64_t *a_eval_launches);
 
+/* Device time in milliseconds (CUDA events on the launching stream, timing
+ * enabled) of the survivor write-out kernel (§8(a) a7: 16 packed 16-byte
+ * records per surviving tuple) of the last synchronous beast_enumerate /
+ * beast_enumerate_to_host on this handle; -1 if that call wrote no list or
+ * timing was off.  *ms: host, out. */
+int beast_last_write_ms(const beast_space *space, float *ms);
+
 #ifdef __cplusplus
 }
 #endif

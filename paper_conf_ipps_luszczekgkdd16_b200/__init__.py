@@ -301,6 +301,11 @@ class Space:
                                               ctypes.byref(n)))
         return int(k.value), float(ms.value), int(n.value)
 
+    def last_write_ms(self):
+        ms = ctypes.c_float(0)
+        _check(_lib.lib().beast_last_write_ms(self.handle, ctypes.byref(ms)))
+        return float(ms.value)
+
     def close(self):
         if self.handle:
             beast_space_destroy(self.handle)

@@ -114,6 +114,7 @@ _sig = {
     "beast_space_set_timing": ([_vp, ctypes.c_int], ctypes.c_int),
     "beast_last_stage_ms": ([_vp, _P(ctypes.c_float)], ctypes.c_int),
     "beast_last_launches": ([_vp, _u64p, _P(ctypes.c_float), _u64p], ctypes.c_int),
+    "beast_last_write_ms": ([_vp, ctypes.POINTER(ctypes.c_float)], ctypes.c_int),
 }
 for _name, (_args, _res) in _sig.items():
     _f = getattr(_L, _name)
