@@ -537,16 +537,34 @@ def ir_measure(beast, desc, stream, flush, canonical_ms, reps=3):
             "note": "generic IR engine (NVRTC-compiled, level-wise) on the same space; counting pass"}
 
 
+def _cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
+
+
 def cpu_baseline(desc):
+    """The oracle nest on this host (SURVEY §8(d) "oracle timing beside it"):
+    all cores (OpenMP over dim_m; the reported value) and one thread."""
     import oracle
     cores = os.cpu_count() or 1
     t = time.perf_counter()
     r = oracle.nest(desc, threads=cores, digest=False)
     dt = time.perf_counter() - t
+    t = time.perf_counter()
+    r1 = oracle.nest(desc, threads=1, digest=False)
+    dt1 = time.perf_counter() - t
+    assert r1["survivors"] == r["survivors"]
     pts = sum(r["visits"])
     return {"value": pts / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
             "sample": "whole space once (%d points, %.1f s wall on %d threads), canonical nest" % (pts, dt, cores),
-            "survivors_per_s": r["survivors"] / dt}
+            "survivors_per_s": r["survivors"] / dt,
+            "single_thread": {"value": pts / dt1, "unit": UNIT, "s": dt1},
+            "cpu": _cpu_model()}
 
 
 if __name__ == "__main__":
