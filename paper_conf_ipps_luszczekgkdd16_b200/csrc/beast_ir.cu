@@ -27,6 +27,7 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <map>
 #include <mutex>
@@ -185,7 +186,8 @@ struct beast_ir {
     std::string err;
     int device = -1;
     cudaLibrary_t lib = nullptr;
-    std::vector<cudaKernel_t> k_count, k_emit;   // per level
+    std::vector<cudaKernel_t> k_count, k_emit;     // per level, warp per parent
+    std::vector<cudaKernel_t> k_tcount, k_temit;   // per level, thread per parent
     cudaKernel_t k_root = nullptr, k_tiles = nullptr, k_top = nullptr,
                  k_add = nullptr;
     int sm_count = 148;
@@ -403,6 +405,55 @@ std::string generate(const beast_ir *ir) {
         snprintf(buf, sizeof(buf), "                ir_row_[%d] = ir_lo_ + (i64)ir_i_ * ir_st_;\n", k);
         s += buf;
         s += "            }\n            ir_pos_ += __popc(ir_bal_);\n        }\n    }\n}\n";
+        // thread-per-parent variants (many parents with short ranges: a warp
+        // per parent would leave most lanes idle and repeat the parent's
+        // bindings 32 times)
+        const std::string thead =
+            "    const unsigned ir_lane_ = threadIdx.x & 31;\n"
+            "    const u64 ir_t0_ = (u64)blockIdx.x * blockDim.x + threadIdx.x;\n"
+            "    const u64 ir_nt_ = (u64)gridDim.x * blockDim.x;\n";
+        snprintf(buf, sizeof(buf),
+                 "extern \"C\" __global__ void __launch_bounds__(256) ir_tcount_%d(const i64 *ir_par_, u64 ir_npar_, "
+                 "u64 *ir_cnt_, u64 *ir_stats_) {\n", k);
+        s += buf;
+        s += thead + consts;
+        snprintf(buf, sizeof(buf), "    u64 ir_vis_ = 0, ir_rej_[%d];\n    for (int ir_q_ = 0; ir_q_ < %d; ++ir_q_) ir_rej_[ir_q_] = 0;\n",
+                 nck > 0 ? nck : 1, nck);
+        s += buf;
+        s += "    for (u64 ir_p_ = ir_t0_; ir_p_ < ir_npar_; ir_p_ += ir_nt_) {\n" + parent;
+        s += "        ir_vis_ += ir_n_;\n        u64 ir_c_ = 0;\n";
+        s += "        for (u64 ir_i_ = 0; ir_i_ < ir_n_; ++ir_i_) {\n" + point;
+        if (nck) s += "            if (ir_r_ == 0) ++ir_c_; else ir_rej_[ir_r_ - 1] += 1;\n";
+        else s += "            ++ir_c_;\n";
+        s += "        }\n        ir_cnt_[ir_p_] = ir_c_;\n    }\n";
+        snprintf(buf, sizeof(buf), "    ir_vis_ = warp_sum(ir_vis_);\n    if (ir_lane_ == 0 && ir_vis_) atomicAdd(&ir_stats_[%d], ir_vis_);\n", k);
+        s += buf;
+        for (int l = 0; l < nck; ++l) {
+            snprintf(buf, sizeof(buf),
+                     "    { const u64 ir_x_ = warp_sum(ir_rej_[%d]); if (ir_lane_ == 0 && ir_x_) atomicAdd(&ir_stats_[NI + %d], ir_x_); }\n",
+                     l, idx[l]);
+            s += buf;
+        }
+        s += "}\n";
+        snprintf(buf, sizeof(buf),
+                 "extern \"C\" __global__ void __launch_bounds__(256) ir_temit_%d(const i64 *ir_par_, u64 ir_npar_, "
+                 "const u64 *ir_off_, i64 *ir_out_) {\n", k);
+        s += buf;
+        s += thead + consts + "    (void)ir_lane_;\n";
+        s += "    for (u64 ir_p_ = ir_t0_; ir_p_ < ir_npar_; ir_p_ += ir_nt_) {\n" + parent;
+        s += "        u64 ir_pos_ = ir_off_[ir_p_];\n";
+        s += "        for (u64 ir_i_ = 0; ir_i_ < ir_n_; ++ir_i_) {\n" + point;
+        s += "            if (ir_r_ == 0) {\n";
+        snprintf(buf, sizeof(buf), "                i64 *ir_row_ = ir_out_ + ir_pos_ * %du;\n", k + 1);
+        s += buf;
+        for (int j = 0; j < k; ++j) {
+            snprintf(buf, sizeof(buf), "                ir_row_[%d] = %s;\n", j, ir->inames[j].c_str());
+            s += buf;
+        }
+        snprintf(buf, sizeof(buf), "                ir_row_[%d] = %s;\n                ++ir_pos_;\n", k,
+                 ir->inames[k].c_str());
+        s += buf;
+        s += "            }\n        }\n    }\n}\n";
     }
     return s;
 }
@@ -454,9 +505,13 @@ int load(beast_ir *ir) {
     IRCK(cudaLibraryGetKernel(&ir->k_root, ir->lib, "ir_root"));
     ir->k_count.assign(ir->ni, nullptr);
     ir->k_emit.assign(ir->ni, nullptr);
+    ir->k_tcount.assign(ir->ni, nullptr);
+    ir->k_temit.assign(ir->ni, nullptr);
     for (int k = 0; k < ir->ni; ++k) {
         IRCK(cudaLibraryGetKernel(&ir->k_count[k], ir->lib, ("ir_count_" + std::to_string(k)).c_str()));
         IRCK(cudaLibraryGetKernel(&ir->k_emit[k], ir->lib, ("ir_emit_" + std::to_string(k)).c_str()));
+        IRCK(cudaLibraryGetKernel(&ir->k_tcount[k], ir->lib, ("ir_tcount_" + std::to_string(k)).c_str()));
+        IRCK(cudaLibraryGetKernel(&ir->k_temit[k], ir->lib, ("ir_temit_" + std::to_string(k)).c_str()));
     }
     IRCK(cudaLibraryGetKernel(&ir->k_tiles, ir->lib, "ir_scan_tiles"));
     IRCK(cudaLibraryGetKernel(&ir->k_top, ir->lib, "ir_scan_top"));
@@ -524,14 +579,19 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
     int rc = BEAST_OK;
     unsigned long long total = 0;
     const unsigned grid = (unsigned)ir->sm_count * 8;
+    // thread per parent once the parents outnumber the resident threads many
+    // times over (BEAST_IR_THREAD_MIN, default 64 x 8 CTAs x 256 threads per SM)
+    unsigned long long thread_min = 64ull * grid * 256;
+    if (const char *e = getenv("BEAST_IR_THREAD_MIN")) thread_min = strtoull(e, nullptr, 10);
     for (int k = 0; k < NI && n_par; ++k) {
+        const bool tmode = n_par >= thread_min;
         unsigned long long *cnt = nullptr, *off = nullptr;
         IRCK(cudaMallocAsync((void **)&cnt, (n_par + 1) * 8, st));
         IRCK(cudaMallocAsync((void **)&off, (n_par + 1) * 8, st));
         {
             const long long *pc = par;
             void *a[] = {(void *)&pc, (void *)&n_par, (void *)&cnt, (void *)&stats};
-            rc = launch(ir, ir->k_count[k], grid, 256, st, a);
+            rc = launch(ir, tmode ? ir->k_tcount[k] : ir->k_count[k], grid, 256, st, a);
         }
         if (rc == BEAST_OK) rc = scan(ir, cnt, n_par, off, st, &total);
         long long *child = nullptr;
@@ -551,7 +611,7 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
             if (rc == BEAST_OK) {
                 const long long *pc = par;
                 void *a[] = {(void *)&pc, (void *)&n_par, (void *)&off, (void *)&child};
-                rc = launch(ir, ir->k_emit[k], grid, 256, st, a);
+                rc = launch(ir, tmode ? ir->k_temit[k] : ir->k_emit[k], grid, 256, st, a);
             }
         }
         cudaFreeAsync(cnt, st);

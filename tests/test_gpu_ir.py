@@ -100,3 +100,36 @@ def test_capacity_error(beast):
         rc = beast._lib.lib().beast_ir_enumerate(sp.handle, None, ctypes.c_void_p(out.data_ptr()), n - 1,
                                                  ctypes.byref(w), None, None)
         assert rc == beast.BEAST_ERR_CAPACITY and w.value == n
+
+
+class _ThreadMode:
+    """Force the thread-per-parent kernels on every level (BEAST_IR_THREAD_MIN
+    = 0; read by each run) -- by default they serve only levels with many
+    parents, which the small parity spaces never reach."""
+
+    def __enter__(self):
+        self.old = os.environ.get("BEAST_IR_THREAD_MIN")
+        os.environ["BEAST_IR_THREAD_MIN"] = "0"
+
+    def __exit__(self, *exc):
+        if self.old is None:
+            os.environ.pop("BEAST_IR_THREAD_MIN", None)
+        else:
+            os.environ["BEAST_IR_THREAD_MIN"] = self.old
+
+
+@pytest.mark.parametrize("name", sorted(ir_specs.toy_specs()))
+def test_toy_specs_thread_per_parent(beast, name):
+    with _ThreadMode():
+        test_toy_specs(beast, name)
+
+
+@pytest.mark.parametrize("p", bi.PRECISIONS)
+def test_gemm_ir_tiny_thread_per_parent(beast, p):
+    with _ThreadMode():
+        _gemm(beast, bi.tiny(p, 0, 1))
+
+
+def test_gemm_ir_medium_thread_per_parent(beast):
+    with _ThreadMode():
+        test_gemm_ir_medium_against_ir_oracle(beast)
