@@ -320,6 +320,32 @@ def main():
         got = beast.beast_wait(pipe_sp[k].handle, pipe_st[k])
         assert got == st_local["survivors"], (got, st_local["survivors"])
     e2e_step = 1e3 * (time.perf_counter() - t) / n_pipe
+    # Informational (not the reported value): device-only passes of the same
+    # handles overlapped on their streams (each still preceded by its own L2
+    # flush): how much of one pass's latency-bound phases another pass's
+    # compute fills.  The reported value stays the one-pass-at-a-time rate.
+    overlapped = None
+    if world == 1:
+        pipe_out = [out] + [torch.empty_like(out) for _ in range(NPIPE - 1)]
+        for k in range(NPIPE):
+            beast.beast_enumerate(pipe_sp[k].handle, pipe_out[k], rank, world, pipe_st[k])
+        torch.cuda.synchronize()
+        t = time.perf_counter()
+        for i in range(n_pipe):
+            k = i % NPIPE
+            if i >= NPIPE:
+                beast.beast_wait(pipe_sp[k].handle, pipe_st[k])
+            with torch.cuda.stream(pipe_st[k]):
+                pipe_flush[k].zero_()
+            beast.beast_enumerate_async(pipe_sp[k].handle, pipe_out[k], rank, world, pipe_st[k])
+        for k in range(NPIPE):
+            assert beast.beast_wait(pipe_sp[k].handle, pipe_st[k]) == st_local["survivors"]
+        ov_ms = 1e3 * (time.perf_counter() - t) / n_pipe
+        overlapped = {"handles": NPIPE, "ms_per_step": ov_ms, "value": n_canon / (ov_ms / 1e3),
+                      "note": "informational: %d passes of the space in flight on %d streams (each with its "
+                              "own L2 flush), host wall clock; the reported value is one pass at a time"
+                              % (NPIPE, NPIPE)}
+        del pipe_out
     for x in extra:
         x.close()
     # the bound of the pipelined e2e: one plain device -> pinned host copy of
@@ -434,6 +460,7 @@ def main():
                     "unpipelined": {"value": n_canon / (e2e_sync_step / 1e3), "ms_per_step": e2e_sync_step,
                                     "how": "beast_enumerate_to_host (synchronous), median step"}},
             "write_out": write_out,
+            "overlapped_passes": overlapped,
             "gpu_launches": launches,
             "clocks": clk,
             "cpu_baseline": cpu,
