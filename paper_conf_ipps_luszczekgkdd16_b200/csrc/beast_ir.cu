@@ -188,6 +188,7 @@ struct beast_ir {
     cudaLibrary_t lib = nullptr;
     std::vector<cudaKernel_t> k_count, k_emit;     // per level, warp per parent
     std::vector<cudaKernel_t> k_tcount, k_temit;   // per level, thread per parent
+    std::vector<cudaKernel_t> k_fcount, k_femit;   // levels k and k + 1 fused (k without constraints), else null
     cudaKernel_t k_root = nullptr, k_tiles = nullptr, k_top = nullptr,
                  k_add = nullptr;
     int sm_count = 148;
@@ -455,6 +456,90 @@ std::string generate(const beast_ir *ir) {
         s += buf;
         s += "            }\n        }\n    }\n}\n";
     }
+    // Fused pairs (k, k + 1) for a level k without constraints: one thread per
+    // parent runs both loops (the level-(k+1) range re-evaluated per value of
+    // k), so the level-k rows are never materialised -- the engine takes them
+    // when a level without constraints has many parents.
+    for (int k = 0; k + 1 < ir->ni; ++k) {
+        bool free_k = true;
+        for (size_t j = 0; j < ir->kexpr.size(); ++j) free_k = free_k && ir->klev[j] != k;
+        if (!free_k) continue;
+        std::vector<int> idx;
+        const std::string cons = constraints_at(k + 1, "                ", &idx);
+        const int nck = (int)idx.size();
+        std::string parent;
+        for (int j = 0; j < k; ++j) {
+            snprintf(buf, sizeof(buf), "        const i64 %s = ir_par_[ir_p_ * %d + %d]; (void)%s;\n",
+                     ir->inames[j].c_str(), k, j, ir->inames[j].c_str());
+            parent += buf;
+        }
+        parent += derived_at(-1, k - 1, "        ");
+        parent += "        const i64 ir_lo_ = (i64)(" + ir->istart[k] + "), ir_hi_ = (i64)(" + ir->istop[k] +
+                  "), ir_st_ = (i64)(" + ir->istep[k] + ");\n";
+        parent += "        const u64 ir_n_ = ir_st_ == 0 ? 0ull : ir_trip(ir_lo_, ir_hi_, ir_st_);\n";
+        std::string outer;   // value of k, its derived variables, the range of k + 1
+        outer += "            const i64 " + ir->inames[k] + " = ir_lo_ + (i64)ir_i_ * ir_st_; (void)" +
+                 ir->inames[k] + ";\n";
+        outer += derived_at(k, k, "            ");
+        outer += "            const i64 ir_lo2_ = (i64)(" + ir->istart[k + 1] + "), ir_hi2_ = (i64)(" +
+                 ir->istop[k + 1] + "), ir_st2_ = (i64)(" + ir->istep[k + 1] + ");\n";
+        outer += "            const u64 ir_n2_ = ir_st2_ == 0 ? 0ull : ir_trip(ir_lo2_, ir_hi2_, ir_st2_);\n";
+        std::string inner;
+        inner += "                const i64 " + ir->inames[k + 1] + " = ir_lo2_ + (i64)ir_j_ * ir_st2_; (void)" +
+                 ir->inames[k + 1] + ";\n";
+        inner += derived_at(k + 1, k + 1, "                ");
+        inner += "                int ir_r_ = 0;\n" + cons;
+        const std::string thead =
+            "    const unsigned ir_lane_ = threadIdx.x & 31;\n"
+            "    const u64 ir_t0_ = (u64)blockIdx.x * blockDim.x + threadIdx.x;\n"
+            "    const u64 ir_nt_ = (u64)gridDim.x * blockDim.x;\n";
+        snprintf(buf, sizeof(buf),
+                 "extern \"C\" __global__ void __launch_bounds__(256) ir_fcount_%d(const i64 *ir_par_, u64 ir_npar_, "
+                 "u64 *ir_cnt_, u64 *ir_stats_) {\n", k);
+        s += buf;
+        s += thead + consts;
+        snprintf(buf, sizeof(buf),
+                 "    u64 ir_vis_ = 0, ir_vis2_ = 0, ir_rej_[%d];\n    for (int ir_q_ = 0; ir_q_ < %d; ++ir_q_) ir_rej_[ir_q_] = 0;\n",
+                 nck > 0 ? nck : 1, nck);
+        s += buf;
+        s += "    for (u64 ir_p_ = ir_t0_; ir_p_ < ir_npar_; ir_p_ += ir_nt_) {\n" + parent;
+        s += "        ir_vis_ += ir_n_;\n        u64 ir_c_ = 0;\n";
+        s += "        for (u64 ir_i_ = 0; ir_i_ < ir_n_; ++ir_i_) {\n" + outer;
+        s += "            ir_vis2_ += ir_n2_;\n";
+        s += "            for (u64 ir_j_ = 0; ir_j_ < ir_n2_; ++ir_j_) {\n" + inner;
+        if (nck) s += "                if (ir_r_ == 0) ++ir_c_; else ir_rej_[ir_r_ - 1] += 1;\n";
+        else s += "                ++ir_c_;\n";
+        s += "            }\n        }\n        ir_cnt_[ir_p_] = ir_c_;\n    }\n";
+        snprintf(buf, sizeof(buf),
+                 "    ir_vis_ = warp_sum(ir_vis_);\n    if (ir_lane_ == 0 && ir_vis_) atomicAdd(&ir_stats_[%d], ir_vis_);\n"
+                 "    ir_vis2_ = warp_sum(ir_vis2_);\n    if (ir_lane_ == 0 && ir_vis2_) atomicAdd(&ir_stats_[%d], ir_vis2_);\n",
+                 k, k + 1);
+        s += buf;
+        for (int l = 0; l < nck; ++l) {
+            snprintf(buf, sizeof(buf),
+                     "    { const u64 ir_x_ = warp_sum(ir_rej_[%d]); if (ir_lane_ == 0 && ir_x_) atomicAdd(&ir_stats_[NI + %d], ir_x_); }\n",
+                     l, idx[l]);
+            s += buf;
+        }
+        s += "}\n";
+        snprintf(buf, sizeof(buf),
+                 "extern \"C\" __global__ void __launch_bounds__(256) ir_femit_%d(const i64 *ir_par_, u64 ir_npar_, "
+                 "const u64 *ir_off_, i64 *ir_out_) {\n", k);
+        s += buf;
+        s += thead + consts + "    (void)ir_lane_;\n";
+        s += "    for (u64 ir_p_ = ir_t0_; ir_p_ < ir_npar_; ir_p_ += ir_nt_) {\n" + parent;
+        s += "        u64 ir_pos_ = ir_off_[ir_p_];\n";
+        s += "        for (u64 ir_i_ = 0; ir_i_ < ir_n_; ++ir_i_) {\n" + outer;
+        s += "            for (u64 ir_j_ = 0; ir_j_ < ir_n2_; ++ir_j_) {\n" + inner;
+        s += "                if (ir_r_ == 0) {\n";
+        snprintf(buf, sizeof(buf), "                    i64 *ir_row_ = ir_out_ + ir_pos_ * %du;\n", k + 2);
+        s += buf;
+        for (int j = 0; j <= k + 1; ++j) {
+            snprintf(buf, sizeof(buf), "                    ir_row_[%d] = %s;\n", j, ir->inames[j].c_str());
+            s += buf;
+        }
+        s += "                    ++ir_pos_;\n                }\n            }\n        }\n    }\n}\n";
+    }
     return s;
 }
 
@@ -512,6 +597,20 @@ int load(beast_ir *ir) {
         IRCK(cudaLibraryGetKernel(&ir->k_emit[k], ir->lib, ("ir_emit_" + std::to_string(k)).c_str()));
         IRCK(cudaLibraryGetKernel(&ir->k_tcount[k], ir->lib, ("ir_tcount_" + std::to_string(k)).c_str()));
         IRCK(cudaLibraryGetKernel(&ir->k_temit[k], ir->lib, ("ir_temit_" + std::to_string(k)).c_str()));
+    }
+    ir->k_fcount.assign(ir->ni, nullptr);
+    ir->k_femit.assign(ir->ni, nullptr);
+    for (int k = 0; k + 1 < ir->ni; ++k) {
+        // fuse (k, k + 1) where level k has no constraints and level k + 1
+        // filters (or is the deepest): its rows are the ones materialised
+        bool free_k = true, filters = k + 2 == ir->ni;
+        for (size_t j = 0; j < ir->kexpr.size(); ++j) {
+            free_k = free_k && ir->klev[j] != k;
+            filters = filters || ir->klev[j] == k + 1;
+        }
+        if (!free_k || !filters) continue;
+        IRCK(cudaLibraryGetKernel(&ir->k_fcount[k], ir->lib, ("ir_fcount_" + std::to_string(k)).c_str()));
+        IRCK(cudaLibraryGetKernel(&ir->k_femit[k], ir->lib, ("ir_femit_" + std::to_string(k)).c_str()));
     }
     IRCK(cudaLibraryGetKernel(&ir->k_tiles, ir->lib, "ir_scan_tiles"));
     IRCK(cudaLibraryGetKernel(&ir->k_top, ir->lib, "ir_scan_top"));
@@ -583,27 +682,33 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
     // times over (BEAST_IR_THREAD_MIN, default 64 x 8 CTAs x 256 threads per SM)
     unsigned long long thread_min = 64ull * grid * 256;
     if (const char *e = getenv("BEAST_IR_THREAD_MIN")) thread_min = strtoull(e, nullptr, 10);
-    for (int k = 0; k < NI && n_par; ++k) {
+    // levels k, k + 1 fused (level k has no constraints) once level k has
+    // this many parents (BEAST_IR_FUSE_MIN, default 8 x 8 CTAs x 256 threads per SM)
+    unsigned long long fuse_min = 8ull * grid * 256;
+    if (const char *e = getenv("BEAST_IR_FUSE_MIN")) fuse_min = strtoull(e, nullptr, 10);
+    for (int k = 0; k < NI && n_par;) {
+        const bool fused = ir->k_fcount[k] != nullptr && n_par >= fuse_min;
         const bool tmode = n_par >= thread_min;
+        const int k_last = fused ? k + 1 : k;   // deepest level of this step
         unsigned long long *cnt = nullptr, *off = nullptr;
         IRCK(cudaMallocAsync((void **)&cnt, (n_par + 1) * 8, st));
         IRCK(cudaMallocAsync((void **)&off, (n_par + 1) * 8, st));
         {
             const long long *pc = par;
             void *a[] = {(void *)&pc, (void *)&n_par, (void *)&cnt, (void *)&stats};
-            rc = launch(ir, tmode ? ir->k_tcount[k] : ir->k_count[k], grid, 256, st, a);
+            rc = launch(ir, fused ? ir->k_fcount[k] : tmode ? ir->k_tcount[k] : ir->k_count[k], grid, 256, st, a);
         }
         if (rc == BEAST_OK) rc = scan(ir, cnt, n_par, off, st, &total);
         long long *child = nullptr;
-        const bool last = k == NI - 1;
+        const bool last = k_last == NI - 1;
         if (rc == BEAST_OK && (!last || emit_last) && total) {
             if (last) {
                 if (total > capacity) rc = BEAST_ERR_CAPACITY;
                 else child = out;
             } else {
-                const cudaError_t e = cudaMallocAsync((void **)&child, total * (unsigned long long)(k + 1) * 8, st);
+                const cudaError_t e = cudaMallocAsync((void **)&child, total * (unsigned long long)(k_last + 1) * 8, st);
                 if (e != cudaSuccess) {
-                    ir->err = "out of device memory for level " + std::to_string(k) + " (" + std::to_string(total) +
+                    ir->err = "out of device memory for level " + std::to_string(k_last) + " (" + std::to_string(total) +
                               " tuples)";
                     rc = BEAST_ERR_WORKSPACE;
                 }
@@ -611,7 +716,7 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
             if (rc == BEAST_OK) {
                 const long long *pc = par;
                 void *a[] = {(void *)&pc, (void *)&n_par, (void *)&off, (void *)&child};
-                rc = launch(ir, tmode ? ir->k_temit[k] : ir->k_emit[k], grid, 256, st, a);
+                rc = launch(ir, fused ? ir->k_femit[k] : tmode ? ir->k_temit[k] : ir->k_emit[k], grid, 256, st, a);
             }
         }
         cudaFreeAsync(cnt, st);
@@ -623,6 +728,7 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
             if (child && child != out) cudaFreeAsync(child, st);
             break;
         }
+        k = k_last + 1;
     }
     if (NI == 0) total = pruned ? 0 : 1;
     std::vector<unsigned long long> h(NI + NC);

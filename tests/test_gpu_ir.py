@@ -102,34 +102,47 @@ def test_capacity_error(beast):
         assert rc == beast.BEAST_ERR_CAPACITY and w.value == n
 
 
-class _ThreadMode:
-    """Force the thread-per-parent kernels on every level (BEAST_IR_THREAD_MIN
-    = 0; read by each run) -- by default they serve only levels with many
+class _Env:
+    """Force the engine's alternative kernel shapes (read by each run): the
+    thread-per-parent kernels on every level (BEAST_IR_THREAD_MIN = 0) and/or
+    the fused two-level kernels wherever a level has no constraints
+    (BEAST_IR_FUSE_MIN = 0) -- by default they serve only levels with many
     parents, which the small parity spaces never reach."""
 
+    MODES = {"thread": {"BEAST_IR_THREAD_MIN": "0"},
+             "fused": {"BEAST_IR_FUSE_MIN": "0"},
+             "fused_thread": {"BEAST_IR_THREAD_MIN": "0", "BEAST_IR_FUSE_MIN": "0"}}
+
+    def __init__(self, mode):
+        self.vars = self.MODES[mode]
+
     def __enter__(self):
-        self.old = os.environ.get("BEAST_IR_THREAD_MIN")
-        os.environ["BEAST_IR_THREAD_MIN"] = "0"
+        self.old = {k: os.environ.get(k) for k in self.vars}
+        os.environ.update(self.vars)
 
     def __exit__(self, *exc):
-        if self.old is None:
-            os.environ.pop("BEAST_IR_THREAD_MIN", None)
-        else:
-            os.environ["BEAST_IR_THREAD_MIN"] = self.old
+        for k, v in self.old.items():
+            if v is None:
+                os.environ.pop(k, None)
+            else:
+                os.environ[k] = v
 
 
+@pytest.mark.parametrize("mode", sorted(_Env.MODES))
 @pytest.mark.parametrize("name", sorted(ir_specs.toy_specs()))
-def test_toy_specs_thread_per_parent(beast, name):
-    with _ThreadMode():
+def test_toy_specs_kernel_shapes(beast, name, mode):
+    with _Env(mode):
         test_toy_specs(beast, name)
 
 
+@pytest.mark.parametrize("mode", sorted(_Env.MODES))
 @pytest.mark.parametrize("p", bi.PRECISIONS)
-def test_gemm_ir_tiny_thread_per_parent(beast, p):
-    with _ThreadMode():
+def test_gemm_ir_tiny_kernel_shapes(beast, p, mode):
+    with _Env(mode):
         _gemm(beast, bi.tiny(p, 0, 1))
 
 
-def test_gemm_ir_medium_thread_per_parent(beast):
-    with _ThreadMode():
+@pytest.mark.parametrize("mode", sorted(_Env.MODES))
+def test_gemm_ir_medium_kernel_shapes(beast, mode):
+    with _Env(mode):
         test_gemm_ir_medium_against_ir_oracle(beast)
