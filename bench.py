@@ -430,7 +430,7 @@ def main():
         clk = clocks.summary()
         cpu = None
         if world == 1 and not args.no_cpu_baseline:
-            cpu = cpu_baseline(desc)
+            cpu = cpu_baseline(desc, n_canon)
         line = {
             "metric": METRIC, "value": n_canon / (ms / 1e3), "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
@@ -574,23 +574,42 @@ def _cpu_model():
     return None
 
 
-def cpu_baseline(desc):
+def cpu_baseline(desc, n_canon=None, budget_points=2.0e10):
     """The oracle nest on this host (SURVEY §8(d) "oracle timing beside it"):
-    all cores (OpenMP over dim_m; the reported value) and one thread."""
+    all cores (OpenMP over dim_m; the reported value) and one thread.  Bounded
+    (the contract's 10-30 s of CPU work): a space of more than budget_points
+    canonical points is sampled as its canonical prefix dim_m <= D (all inner
+    loops), and the one-thread run is bounded the same way to ~20 s."""
     import oracle
     cores = os.cpu_count() or 1
+    dmx = oracle.resolve(desc)["dim_m_max"]
+
+    def sampled(d):
+        return desc if d >= dmx else dict(desc, dim_m_max=d)
+
+    d = dmx
+    if n_canon and n_canon > budget_points:
+        d = max(1, int(dmx * budget_points / n_canon))
     t = time.perf_counter()
-    r = oracle.nest(desc, threads=cores, digest=False)
+    r = oracle.nest(sampled(d), threads=cores, digest=False)
     dt = time.perf_counter() - t
-    t = time.perf_counter()
-    r1 = oracle.nest(desc, threads=1, digest=False)
-    dt1 = time.perf_counter() - t
-    assert r1["survivors"] == r["survivors"]
     pts = sum(r["visits"])
+    what = "whole space once" if d >= dmx else "canonical prefix dim_m <= %d of the space" % d
+    # one thread: ~20 s at most (rate scaled from the all-core run)
+    d1 = d
+    est = dt * cores
+    if est > 20.0:
+        d1 = max(1, int(d * 20.0 / est))
+    t = time.perf_counter()
+    r1 = oracle.nest(sampled(d1), threads=1, digest=False)
+    dt1 = time.perf_counter() - t
+    if d1 == d:
+        assert r1["survivors"] == r["survivors"]
     return {"value": pts / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
-            "sample": "whole space once (%d points, %.1f s wall on %d threads), canonical nest" % (pts, dt, cores),
+            "sample": "%s (%d points, %.1f s wall on %d threads), canonical nest" % (what, pts, dt, cores),
             "survivors_per_s": r["survivors"] / dt,
-            "single_thread": {"value": pts / dt1, "unit": UNIT, "s": dt1},
+            "single_thread": {"value": sum(r1["visits"]) / dt1, "unit": UNIT, "s": dt1,
+                              "sample": "whole space" if d1 >= dmx else "canonical prefix dim_m <= %d" % d1},
             "cpu": _cpu_model()}
 
 
