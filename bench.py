@@ -574,37 +574,38 @@ def _cpu_model():
     return None
 
 
-def cpu_baseline(desc, n_canon=None, budget_points=2.0e10):
+def cpu_baseline(desc, n_canon=None, budget_s=10.0):
     """The oracle nest on this host (SURVEY §8(d) "oracle timing beside it"):
     all cores (OpenMP over dim_m; the reported value) and one thread.  Bounded
-    (the contract's 10-30 s of CPU work): a space of more than budget_points
-    canonical points is sampled as its canonical prefix dim_m <= D (all inner
-    loops), and the one-thread run is bounded the same way to ~20 s."""
+    for the one-thread rate: the whole space if it takes at most budget_s,
+    else the canonical prefix dim_m <= D with D doubled from 1 while a run
+    stays under budget_s (the work is far from uniform in dim_m, so D is
+    found by measurement)."""
     import oracle
     cores = os.cpu_count() or 1
     dmx = oracle.resolve(desc)["dim_m_max"]
 
-    def sampled(d):
-        return desc if d >= dmx else dict(desc, dim_m_max=d)
+    def run(threads):
+        d, best = 1, None
+        while True:
+            dd = min(d, dmx)
+            t = time.perf_counter()
+            r = oracle.nest(desc if dd >= dmx else dict(desc, dim_m_max=dd), threads=threads, digest=False)
+            dt = time.perf_counter() - t
+            best = (dd, r, dt)
+            if dd >= dmx or dt * 2.5 > budget_s:   # the next doubling would overrun the budget
+                return best
+            d *= 2
 
-    d = dmx
-    if n_canon and n_canon > budget_points:
-        d = max(1, int(dmx * budget_points / n_canon))
+    # all cores: the whole space (the OpenMP loop is over dim_m, so a dim_m
+    # prefix would starve the cores; the headline takes ~0.5 s, the largest
+    # configuration ~70 s); one thread: the doubling prefix
     t = time.perf_counter()
-    r = oracle.nest(sampled(d), threads=cores, digest=False)
-    dt = time.perf_counter() - t
+    r = oracle.nest(desc, threads=cores, digest=False)
+    d, dt = dmx, time.perf_counter() - t
+    d1, r1, dt1 = run(1)
     pts = sum(r["visits"])
     what = "whole space once" if d >= dmx else "canonical prefix dim_m <= %d of the space" % d
-    # one thread: ~20 s at most (rate scaled from the all-core run)
-    d1 = d
-    est = dt * cores
-    if est > 20.0:
-        d1 = max(1, int(d * 20.0 / est))
-    t = time.perf_counter()
-    r1 = oracle.nest(sampled(d1), threads=1, digest=False)
-    dt1 = time.perf_counter() - t
-    if d1 == d:
-        assert r1["survivors"] == r["survivors"]
     return {"value": pts / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
             "sample": "%s (%d points, %.1f s wall on %d threads), canonical nest" % (what, pts, dt, cores),
             "survivors_per_s": r["survivors"] / dt,
