@@ -133,6 +133,13 @@ def widened(blk_max=256, device="k40c", precision="D", trans_a=0, trans_b=0):
                       bounds=(0, 0, blk_max, blk_max, blk_max))
 
 
+def maxbound(device="k40c", precision="D", trans_a=0, trans_b=0):
+    """Edge case: all five iterator bounds at 4095, the largest the packed
+    12-bit record fields (and the library's validation) admit."""
+    dev = K40C_DEVICE if device == "k40c" else B200_DEVICE
+    return make_space(dev, precision, trans_a, trans_b, bounds=4095)
+
+
 NAMED = {
     "tiny": lambda: tiny("D"),
     "micro": lambda: micro("C"),

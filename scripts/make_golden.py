@@ -43,6 +43,9 @@ def spaces():
     for p in ("D", "Z", "C", "S"):
         for ta, tb in bi.TRANSPOSES:
             out["b200_%s_%d%d" % (p, ta, tb)] = bi.b200(p, ta, tb)
+    out["maxbound_k40c_D_00"] = bi.maxbound("k40c", "D")
+    out["maxbound_k40c_Z_11"] = bi.maxbound("k40c", "Z", 1, 1)
+    out["maxbound_b200_D_00"] = bi.maxbound("b200", "D")
     return out
 
 

@@ -97,7 +97,8 @@ def test_headline_bit_exact(beast):
 GOLDEN_BIG = ["k40c_%s_%d%d" % (p, a, b) for p in bi.PRECISIONS for a, b in bi.TRANSPOSES] + \
              ["b200_%s_%d%d" % (p, a, b) for p in bi.PRECISIONS for a, b in bi.TRANSPOSES] + \
              ["widened%d_%s_D_00" % (w, d) for w in (64, 256, 512) for d in ("k40c", "b200")] + \
-             ["b200_48k_D_00", "b200_48k_S_00"]
+             ["b200_48k_D_00", "b200_48k_S_00"] + \
+             ["maxbound_k40c_D_00", "maxbound_k40c_Z_11", "maxbound_b200_D_00"]
 
 
 @pytest.mark.parametrize("key", GOLDEN_BIG)
