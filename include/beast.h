@@ -29,9 +29,11 @@
  *     handle is not safe for concurrent calls; separate handles are
  *     independent.  Device calls run on the CUDA device current at call
  *     time, which must not change over the handle's life.
- *   - rank / world select a shard: the contiguous canonical range of L7
- *     prefixes whose cumulative enumeration work falls in
- *     [W*rank/world, W*(rank+1)/world).  The global survivor list is the
+ *   - rank / world select a shard: the contiguous canonical range of L4
+ *     survivors (dim_m, dim_n, blk_m, blk_n) whose cumulative estimated
+ *     enumeration work falls in [W*rank/world, W*(rank+1)/world), with every
+ *     point below them (L5-L15).  Levels L1-L4 run on every rank; their
+ *     statistics are reported by rank 0 only.  The global survivor list is the
  *     concatenation of the shards in rank order.  world = 1, rank = 0 is the
  *     whole space.  The library never communicates between ranks.
  *   - There is no CPU fallback: every call that enumerates needs a CUDA

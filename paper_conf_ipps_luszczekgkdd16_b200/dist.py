@@ -1,8 +1,9 @@
 """Multi-GPU combine (§X-B: parallelise the
 outermost loop nests).
 
-One process per GPU (torchrun).  Every rank runs the replicated prefix stage
-and enumerates its own contiguous canonical shard of L7 prefixes through the
+One process per GPU (torchrun).  Every rank runs levels L1-L4 of the prefix
+stage (replicated) and enumerates its own contiguous canonical shard -- a
+work-balanced range of L4 survivors and everything below them -- through the
 C ABI (beast_enumerate(rank, world)); the library never communicates.  This
 module does the one exchange the method has:
 
