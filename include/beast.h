@@ -176,8 +176,11 @@ int beast_limits_resolve(beast_device_limits *limits);
 /* Create a space description.  settings / bounds may be NULL (trans 0/0,
  * thresholds 256/2; default bounds).  Validates and resolves the inputs on
  * the host only; no device work.  BEAST_ERR_UNSUPPORTED if a bound exceeds
- * 4095 (the 12-bit record fields), if max_threads_per_block > 65535, or if a
- * limit is non-positive where the paper divides by it; BEAST_ERR_INVALID_ARGUMENT
+ * 4095 (the 12-bit record fields), if max_threads_per_block > 65535,
+ * max_blocks_per_multi_processor > 65534, float_size > 1024,
+ * min_threads_per_multi_processor > 2^30 or min_fmas_per_load > 2^20 (the
+ * ranges the packed words and the integer predicate arithmetic cover), or if
+ * a limit is non-positive where the paper divides by it; BEAST_ERR_INVALID_ARGUMENT
  * for NULL limits/out or a bad precision.  *out: owned by the caller, release
  * with beast_space_destroy. */
 int beast_space_create(const beast_device_limits *limits, beast_precision precision,
