@@ -38,7 +38,7 @@ def launches(tag, wl):
     names = [r[ki].split("(")[0].replace("void ", "").replace("beast::", "") for r in data]
     vals = [float(r[vi].replace(",", "")) for r in data]
     # one step = the last run of launches starting at the first-level count kernel
-    starts = [i for i, n in enumerate(names) if n.startswith(("k_seg_count<", "k_seg_level<")) and "PairsSeg" in n]
+    starts = [i for i, n in enumerate(names) if n.startswith(("k_seg_count<", "k_seg_level<")) and ("PairsSeg" in n or "PairRowsSeg" in n)]
     bounds = list(zip(starts, starts[1:] + [len(names)]))
     # the last canonical pass (the bench also times the factorised path)
     a, b = [(a, b) for a, b in bounds if any(n.startswith("k_eval<") for n in names[a:b])][-1]
