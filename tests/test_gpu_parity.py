@@ -300,3 +300,31 @@ def test_host_async_pipelined_handles(beast, golden_expected):
     finally:
         for sp in sps:
             sp.close()
+
+
+@pytest.mark.gpu
+def test_host_async_shards_concatenate(beast, golden_expected):
+    """beast_enumerate_to_host_async on shard handles (virtual ranks of 3):
+    the host lists concatenated in rank order are the world-1 list."""
+    import torch
+    e = golden_expected["k40c_D_00"]
+    world = 3
+    sps = [beast.Space.from_desc(bi.headline()) for _ in range(world)]
+    try:
+        hosts, streams = [], []
+        for r, sp in enumerate(sps):
+            n = sp.count(rank=r, world=world)
+            hosts.append(torch.empty((n, 2), dtype=torch.uint64).pin_memory())
+            streams.append(torch.cuda.Stream())
+            assert beast.beast_enumerate_to_host(sp.handle, hosts[r], r, world, streams[r]) == n
+            hosts[r].zero_()
+        for r, sp in enumerate(sps):
+            beast.beast_enumerate_to_host_async(sp.handle, hosts[r], r, world, streams[r])
+        for r, sp in enumerate(sps):
+            assert beast.beast_wait(sp.handle, streams[r]) == hosts[r].shape[0]
+        full = torch.cat(hosts).cuda()
+        assert full.shape[0] == e["survivors"]
+        assert "0x%016x" % beast.beast_digest(full) == e["digest"]
+    finally:
+        for sp in sps:
+            sp.close()
