@@ -410,7 +410,7 @@ def main():
                          "achieved_GBps": w_gbs, "peak_GBps": peaks["hbm_gbs"], "frac": w_gbs / peaks["hbm_gbs"],
                          "peak_source": "MEASURED_PEAKS.json hbm_gbs (%s; a read+write copy rate, the "
                                         "write-only kernel is compared against it)" % peak_src}
-        a_points = stats["visits"][8]          # L9 points: one launch evaluates all of them
+        a_points = st_local["visits"][8]       # this rank's L9 points: its launch evaluates all of them
         # Roofline: every point needs one product and one
         # compare = 2 integer ops.  Peak = issue-bound integer lane rate with
         # 16-bit SIMD (one 32-bit lane instruction carries two 16-bit ops):
@@ -419,7 +419,7 @@ def main():
         sm_count = torch.cuda.get_device_properties(0).multi_processor_count
         lanes = 128                            # integer lane-instructions / clk / SM (4 x 32, ALU + FMA pipes)
         peak_ops = sm_count * lanes * 2 * float(peaks.get("sm_max_mhz", 1965.0)) * 1e6
-        achieved = ops_per_point * a_points / (a_ms / 1e3) / world if a_ms > 0 else 0.0
+        achieved = ops_per_point * a_points / (a_ms / 1e3) if a_ms > 0 else 0.0
         traffic = None
         prof = os.path.join(ROOT, "profiles", "k_eval_traffic.json")
         if os.path.exists(prof):
@@ -443,7 +443,7 @@ def main():
             "roofline": {"bound": "alu", "kernel": "k_eval<A> (L8-L9 A-read grids)",
                          "achieved": achieved / 1e12, "peak": peak_ops / 1e12, "unit": "T int16-ops/s",
                          "frac": achieved / peak_ops if peak_ops else None, "traffic": traffic,
-                         "algorithmic_ops_per_launch": ops_per_point * a_points // world,
+                         "algorithmic_ops_per_launch": ops_per_point * a_points,
                          "avg_launch_ms": a_ms,
                          "peak_source": "%d SMs x %d int lane-instr/clk x 2 (16-bit halves) x sm_max_mhz (%s "
                                         "MEASURED_PEAKS.json); 2 int ops per point" % (sm_count, lanes, peak_src),
