@@ -328,3 +328,28 @@ def test_host_async_shards_concatenate(beast, golden_expected):
     finally:
         for sp in sps:
             sp.close()
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("seed", range(24))
+def test_fuzz_shards_vs_oracle(beast, seed):
+    """Shard rule on fuzz spaces: for a seeded world in 2..9
+    -- often more ranks than L4 survivors, so some shards are empty -- the
+    shards concatenated in rank order are the oracle's list and their
+    statistics sum to the oracle's."""
+    desc = bi.fuzz_space(seed)
+    world = 2 + random.Random(1000 + seed).randrange(8)
+    ref = oracle.nest(desc, records=True)
+    parts, visits, rejected, counts = [], np.zeros(15, np.int64), np.zeros(12, np.int64), 0
+    for r in range(world):
+        got, st, _, n = _run(beast, desc, rank=r, world=world)
+        assert n == len(got)
+        parts.append(got)
+        counts += n
+        visits += np.array(st["visits"], np.int64)
+        rejected += np.array(st["rejected"], np.int64)
+    cat = np.concatenate(parts) if parts else np.zeros((0, 2), np.uint64)
+    want = _oracle_lohi(ref["records"])
+    assert cat.shape == want.shape and np.array_equal(cat, want), (seed, world)
+    assert counts == ref["survivors"]
+    assert list(visits) == ref["visits"] and list(rejected) == ref["rejected"], (seed, world)
