@@ -160,6 +160,141 @@ def named(name: str) -> dict:
     return NAMED[name]()
 
 
+def _log_int(r: random.Random, lo: int, hi: int) -> int:
+    """Integer in [lo, hi], log-uniform (lo >= 1)."""
+    import math
+    return min(hi, max(lo, int(math.exp(r.uniform(math.log(lo), math.log(hi + 1))))))
+
+
+# Admitted ranges of beast_space_create (include/beast.h): the widest values
+# the library accepts.  fuzz_space_wide draws from these.
+ADMITTED = dict(max_threads_per_block=65535, float_size=1024, max_blocks_per_multi_processor=65534,
+                min_threads_per_multi_processor=1 << 30, min_fmas_per_load=1 << 20, bound=4095,
+                int32=(1 << 31) - 1)
+
+
+def fuzz_space_wide(seed: int, attempt: int = 0) -> dict:
+    """Seeded random space over the library's whole admitted range (seeds
+    200-399 of the test plan): max_threads_per_block up to 65535 (so
+    threads_per_block up to 65535), warp_size in {1, ..., 64}, every bound up
+    to 4095, float_size up to 1024, max_blocks_per_multi_processor up to
+    65534, shared-memory / register limits and max_registers_per_thread up
+    to 2^31 - 1, thresholds min_threads up to 2^30 and min_fmas up to 2^20.
+    Three regimes, so that the draws also leave survivors: "hostile" (every
+    value log-uniform over its whole range, the cap one time in five),
+    "friendly" (limits drawn from the permissive upper part of their ranges,
+    small thresholds) and "big_t" (friendly, with max_threads_per_block >=
+    2048 and bounds 16-512, where threads_per_block > 1024 survives).
+    `attempt` re-draws the same seed (scripts/make_wide_fuzz.py keeps the
+    first attempt whose canonical nest the oracle finishes within its
+    budget)."""
+    r = random.Random(seed * 7919 + attempt * 104729 + 17)
+    A = ADMITTED
+    mode = r.choices(("hostile", "friendly", "big_t"), (0.3, 0.3, 0.4))[0]
+
+    def draw(lo, typical, hi):
+        """the cap (1/5), log-uniform over [lo, typical] (2/5) or over the
+        whole admitted range [lo, hi] (2/5)"""
+        u = r.random()
+        if u < 0.2:
+            return hi
+        return _log_int(r, lo, typical if u < 0.6 else hi)
+
+    def high(lo, hi):
+        """the cap (1/2) or log-uniform over [lo, hi]"""
+        return hi if r.random() < 0.5 else _log_int(r, lo, hi)
+
+    warp = r.choice((1, 2, 4, 8, 16, 32, 64))
+    dev = dict(K40C_DEVICE)
+    dev["warp_size"] = warp
+    dev["float_size"] = draw(1, 16, A["float_size"])
+    if mode == "hostile":
+        dev["max_threads_per_block"] = draw(warp, 4096, A["max_threads_per_block"])
+        dev["max_shared_mem_per_block"] = draw(16, 1 << 18, A["int32"])
+        dev["max_shmem_per_multi_processor"] = draw(16, 1 << 18, A["int32"])
+        dev["max_regs_per_block"] = draw(1, 1 << 17, A["int32"])
+        dev["max_registers_per_multi_processor"] = draw(1, 1 << 17, A["int32"])
+        fig9 = dict(max_blocks_per_multi_processor=draw(1, 64, A["max_blocks_per_multi_processor"]),
+                    max_registers_per_thread=draw(1, 256, A["int32"]))
+        bounds = tuple(draw(1, 128, A["bound"]) for _ in range(5))
+        mt = 0 if r.random() < 0.1 else draw(1, 2048, A["min_threads_per_multi_processor"])
+        mf = 0 if r.random() < 0.1 else draw(1, 8, A["min_fmas_per_load"])
+    elif mode == "friendly":
+        dev["max_threads_per_block"] = high(warp, A["max_threads_per_block"])
+        dev["max_shared_mem_per_block"] = high(1 << 16, A["int32"])
+        dev["max_shmem_per_multi_processor"] = high(1 << 16, A["int32"])
+        dev["max_regs_per_block"] = high(1 << 16, A["int32"])
+        dev["max_registers_per_multi_processor"] = high(1 << 16, A["int32"])
+        fig9 = dict(max_blocks_per_multi_processor=high(8, A["max_blocks_per_multi_processor"]),
+                    max_registers_per_thread=high(64, A["int32"]))
+        bounds = tuple(draw(1, 128, A["bound"]) for _ in range(5))
+        u = r.random()
+        mt = 0 if u < 0.2 else A["min_threads_per_multi_processor"] if u < 0.25 else _log_int(r, 1, 2048)
+        u = r.random()
+        mf = 0 if u < 0.2 else A["min_fmas_per_load"] if u < 0.25 else _log_int(r, 1, 8)
+    else:
+        # big_t: few resident blocks and a high occupancy threshold keep
+        # only large threads_per_block (min_threads / max_blocks), few
+        # registers per thread keep blk_m, blk_n near dim_m, dim_n
+        dev["max_threads_per_block"] = high(4096, A["max_threads_per_block"])
+        for k in ("max_shared_mem_per_block", "max_shmem_per_multi_processor", "max_regs_per_block",
+                  "max_registers_per_multi_processor"):
+            dev[k] = A["int32"] if r.random() < 0.7 else _log_int(r, 1 << 22, A["int32"])
+        mb = r.randint(1, 4)
+        fig9 = dict(max_blocks_per_multi_processor=mb, max_registers_per_thread=_log_int(r, 8, 256))
+        bounds = (_log_int(r, 64, 1024), _log_int(r, 64, 1024), _log_int(r, 64, 2048),
+                  _log_int(r, 64, 2048), _log_int(r, 32, 1024))
+        mt = mb * _log_int(r, 1024, max(1024, dev["max_threads_per_block"] // 2))
+        mf = r.randint(0, 1)
+    fig9["max_warps_per_multi_processor"] = r.choice((16, 32, 48, 64))
+    return make_space(dev, r.choice(PRECISIONS), r.randint(0, 1), r.randint(0, 1), bounds=bounds,
+                      min_threads_per_multi_processor=mt, min_fmas_per_load=mf, **fig9)
+
+
+# Edge spaces at the limits beast_space_create admits (include/beast.h):
+# threads_per_block up to 65535, float_size 1024, max_blocks 65534 with the
+# occupancy threshold 2^30, min_fmas 2^20, limits at 2^31 - 1.  Goldens come
+# from scripts/make_golden.py (oracle only).
+_INT32 = (1 << 31) - 1
+_OPEN = dict(K40C_DEVICE, max_threads_per_block=65535, max_shared_mem_per_block=_INT32,
+             max_shmem_per_multi_processor=_INT32, max_regs_per_block=_INT32,
+             max_registers_per_multi_processor=_INT32)
+EXTREME = {
+    # 16384 <= threads_per_block <= 65535, a multiple of 64 (one resident
+    # block must reach the occupancy threshold)
+    "ext_bigT_D_00": lambda: make_space(dict(_OPEN, warp_size=64), "D", 0, 0, bounds=(256, 256, 512, 512, 256),
+                                        min_threads_per_multi_processor=16384, min_fmas_per_load=0,
+                                        max_blocks_per_multi_processor=1, max_registers_per_thread=4),
+    # threads_per_block >= 4096, any multiple of 1, SGEMM (dim_vec 4), both transposes
+    "ext_bigT_S_11": lambda: make_space(dict(_OPEN, warp_size=1), "S", 1, 1, bounds=(128, 128, 256, 256, 64),
+                                        min_threads_per_multi_processor=4096, min_fmas_per_load=1,
+                                        max_blocks_per_multi_processor=1, max_registers_per_thread=8),
+    # float_size 1024 against 2^31 - 1 bytes of shared memory
+    "ext_float1024_C_10": lambda: make_space(dict(_OPEN, max_threads_per_block=4096, float_size=1024), "C", 1, 0,
+                                             bounds=(64, 64, 128, 128, 128),
+                                             max_blocks_per_multi_processor=32, max_registers_per_thread=255),
+    # max_blocks 65534 and min_threads 65534 * 32: need = ceil(min_threads / T)
+    # is 65534 at T = 32 and exceeds max_blocks below it (the saturated
+    # need of the packed L3 row word)
+    "ext_need_edge_D_00": lambda: make_space(dict(_OPEN, warp_size=1, float_size=1), "D", 0, 0,
+                                             bounds=(64, 64, 128, 128, 64),
+                                             min_threads_per_multi_processor=65534 * 32, min_fmas_per_load=0,
+                                             max_blocks_per_multi_processor=65534, max_registers_per_thread=255),
+    # min_threads 2^30 with max_blocks 65534 (threads_per_block >= 16385 needed)
+    "ext_occ_cap_S_01": lambda: make_space(dict(_OPEN, warp_size=1, float_size=1), "S", 0, 1,
+                                           bounds=(256, 256, 512, 512, 64),
+                                           min_threads_per_multi_processor=1 << 30, min_fmas_per_load=0,
+                                           max_blocks_per_multi_processor=65534, max_registers_per_thread=2),
+    # min_fmas 2^20 (every L6 point fails low_fmas)
+    "ext_fmas_cap_D_00": lambda: make_space(K40C_DEVICE, "D", 0, 0, bounds=(64, 64, 256, 256, 256),
+                                            min_fmas_per_load=1 << 20),
+}
+
+
+def extreme(name: str) -> dict:
+    return EXTREME[name]()
+
+
 def fuzz_space(seed: int, max_bound: int = 24) -> dict:
     """Seeded random small space (SURVEY §8(d) fuzz recipe): bounds in
     [1, max_bound]; warp_size in {4, 8, 16, 32}; max_threads_per_block in

@@ -34,9 +34,28 @@ def _divisors(t: int):
     return [x for x in range(1, t + 1) if t % x == 0]
 
 
-def count(space: dict) -> dict:
+def _add_shapes(hist: dict, rows, cols, weight) -> None:
+    """hist[(rows, cols)] += weight, for parallel arrays."""
+    if rows.size == 0:
+        return
+    key = np.stack([rows, cols], axis=1)
+    uk, inv = np.unique(key, axis=0, return_inverse=True)
+    w = np.bincount(inv.ravel(), weights=weight.astype(np.float64), minlength=len(uk))
+    for (a, b), c in zip(uk.tolist(), w.tolist()):
+        if c:
+            hist[(a, b)] = hist.get((a, b), 0) + int(round(c))
+
+
+def count(space: dict, shapes: bool = False) -> dict:
     """Returns dict(visits[15], rejected[12], survivors, prefixes (L7 visits),
-    valid_a (number of (prefix, dim_m_a, dim_n_a) passing a1 and a2))."""
+    valid_a (number of (prefix, dim_m_a, dim_n_a) passing a1 and a2)).
+    shapes=True adds the grid-shape histograms of the L8-L11 loops:
+    a_shapes[(RA_m, RA_n)] = number of L7 prefixes whose A-read grid
+    (dim_m_a in 1..RA_m, dim_n_a in 1..RA_n) has that shape, and
+    b_shapes[(RB_m, RB_n)] = number of valid (prefix, A grid) pairs whose
+    B-read grid has that shape -- sum(RA_m * RA_n * count) is
+    visits[8] and sum(RB_m * RB_n * count) is visits[10]."""
+    a_shapes, b_shapes = {}, {}
     s = resolve(space)
     prec = space["precision"]
     cr = 2 if prec in ("D", "Z") else 1
@@ -125,6 +144,8 @@ def count(space: dict) -> dict:
             rbn = bn if tb == 0 else bkk
             V[7] += nvm * int(ram.sum())
             V[8] += nvm * int((ram * ran).sum())
+            if shapes:
+                _add_shapes(a_shapes, ram, ran, np.full(ram.shape, nvm))
             a1h = np.zeros_like(bm)
             na = np.zeros_like(bm)
             b1h = np.zeros_like(bm)
@@ -152,9 +173,14 @@ def count(space: dict) -> dict:
             R[9] += nvm * int((na * (rbm * rbn - b1h)).sum())
             R[11] += nvm * int((na * (b1h - nb)).sum())
             valid_a += nvm * int(na.sum())
+            if shapes:
+                _add_shapes(b_shapes, rbm, rbn, nvm * na)
             tuples += nvm * int((na * nb).sum())
     V[11] = 2 * tuples
     V[12] = 4 * tuples
     V[13] = 8 * tuples
     V[14] = 16 * tuples
-    return dict(visits=V, rejected=R, survivors=V[14], prefixes=V[6], valid_a=valid_a)
+    out = dict(visits=V, rejected=R, survivors=V[14], prefixes=V[6], valid_a=valid_a)
+    if shapes:
+        out.update(a_shapes=a_shapes, b_shapes=b_shapes)
+    return out

@@ -46,6 +46,8 @@ def spaces():
     out["maxbound_k40c_D_00"] = bi.maxbound("k40c", "D")
     out["maxbound_k40c_Z_11"] = bi.maxbound("k40c", "Z", 1, 1)
     out["maxbound_b200_D_00"] = bi.maxbound("b200", "D")
+    for name in bi.EXTREME:                 # the admitted-range edge spaces
+        out[name] = bi.extreme(name)
     return out
 
 
