@@ -46,6 +46,19 @@ WORKLOADS = {
 # Paper timings of this path (context only):
 PAPER_CONTEXT = {"python_s": 66948, "c_s": 264, "cpu": "Xeon E5-2650 v3, 1 core"}
 
+# Measured packed-scan ceiling (profiles/r02_micro/README.md, scripts/micro/scan.cu:
+# the best 16-pair block body, 8 IMAD + 8 VIADDMNMX, at 64 warps/SM): points
+# per clock per SM.
+SCAN_CEILING_POINTS_PER_CLK_SM = 134.75
+
+
+def config_dict(args, n_canon, survivors):
+    """The `config` object of both arms (same keys and values, so the
+    driver's same-config check compares like with like)."""
+    return {"workload": args.workload, "description": WORKLOADS.get(args.workload, args.workload),
+            "n_canon": n_canon, "survivors": survivors, "parallelism": "dp%d" % args.gpus,
+            "gather": args.gather if args.gpus > 1 else None}
+
 
 def _load_peaks():
     try:
@@ -148,14 +161,20 @@ def run_reference(args):
         n_canon, survivors = sum(r["visits"]), r["survivors"]
     ms = 1e3 * sum(times) / len(times)
     value = n_canon / (ms / 1e3)
+    # the whole workload's size for the config object (the sample may be a prefix)
+    if "prefix" in sample:
+        import oracle.analytic
+        full = oracle.analytic.count(beast_inputs.named(args.workload))
+        cfg_canon, cfg_surv = sum(full["visits"]), full["survivors"]
+    else:
+        cfg_canon, cfg_surv = n_canon, survivors
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
-        "config": {"workload": args.workload, "description": WORKLOADS.get(args.workload, args.workload),
-                   "n_canon": n_canon, "survivors": survivors},
+        "config": config_dict(args, cfg_canon, cfg_surv),
         "survivors_per_s": survivors / (ms / 1e3),
-        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "cpu": _cpu_model(),
                          "sample": "%s (%d points), canonical nest, OpenMP over dim_m" % (sample, n_canon)},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
@@ -180,6 +199,8 @@ def main():
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":
         return run_reference(args)
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return relaunch(args)
 
     import torch
     import torch.distributed as dist
@@ -194,19 +215,24 @@ def main():
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world != args.gpus:
-        world = args.gpus if world == 1 and args.gpus == 1 else world
+        print("bench.py: --gpus %d but WORLD_SIZE=%d ranks were launched" % (args.gpus, world), file=sys.stderr)
+        return 2
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        assert dist.get_world_size() == args.gpus
     desc = beast_inputs.named(args.workload)
     sp = beast.Space.from_desc(desc)
     stream = torch.cuda.current_stream()
 
-    # sizes (and the canonical point count) from one instrumented pass
+    # sizes (and the canonical point count) from one instrumented pass; the
+    # ranks' redundantly computed L1-L4 lists are checked equal by digest
+    # (combine_stats all-gathers l4_digest)
     _, st_local = sp.enumerate(rank=rank, world=world, stats=True)
     stats = bdist.combine_stats(st_local, world)
     n_canon = stats["points"]
     survivors = stats["survivors"]
+    replicas = bdist.check_replicas(sp.last_l4_digest(), world)
 
     out = torch.empty((max(st_local["survivors"], 1), 2), dtype=torch.uint64, device="cuda")
     gathered = torch.empty((max(survivors, 1), 2), dtype=torch.uint64, device="cuda") if rank == 0 else None
@@ -262,6 +288,51 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         total_ms = float(t.item())
     ms = total_ms / args.steps
+
+    # Sharded-resident: the same passes without the gather --
+    # every rank's shard stays in its own HBM (the global list is the
+    # concatenation in rank order); device time per step, max over ranks.
+    sharded = None
+    if world > 1:
+        rev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+               for _ in range(args.steps)]
+        dist.barrier()
+        torch.cuda.synchronize()
+        for i in range(args.steps):
+            flush.zero_()
+            rev[i][0].record(stream)
+            beast.beast_enumerate_async(sp.handle, out, rank, world, stream)
+            rev[i][1].record(stream)
+        assert beast.beast_wait(sp.handle, stream) == st_local["survivors"]
+        torch.cuda.synchronize()
+        t = torch.tensor([sum(a.elapsed_time(b) for a, b in rev) / args.steps], dtype=torch.float64,
+                         device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        sms = float(t.item())
+        sharded = {"ms_per_step": sms, "value": n_canon / (sms / 1e3),
+                   "how": "beast_enumerate_async per rank, no gather (list resident as N shards); "
+                          "CUDA events, max over ranks"}
+
+    # count (beast_count: the same pass without compaction order and
+    # write-out), timed on its own: CUDA events around each synchronous call
+    cnt_ms = []
+    sp.count(rank=rank, world=world, stream=stream)
+    for _ in range(max(3, args.steps // 2)):
+        flush.zero_()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        sp.count(rank=rank, world=world, stream=stream)
+        b.record(stream)
+        b.synchronize()
+        cnt_ms.append(a.elapsed_time(b))
+    c_ms = statistics.median(cnt_ms)
+    if world > 1:
+        t = torch.tensor([c_ms], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        c_ms = float(t.item())
+    count_line = {"ms_per_step": c_ms, "value": n_canon / (c_ms / 1e3), "unit": UNIT,
+                  "how": "beast_count (survivor count only: no canonical placement, no write-out), "
+                         "median of synchronous flushed calls, CUDA events"}
 
     # Roofline: the dominant kernel's launches timed by the library's CUDA
     # events on the launching stream, over K synchronous flushed steps.
@@ -420,6 +491,8 @@ def main():
         lanes = 128                            # integer lane-instructions / clk / SM (4 x 32, ALU + FMA pipes)
         peak_ops = sm_count * lanes * 2 * float(peaks.get("sm_max_mhz", 1965.0)) * 1e6
         achieved = ops_per_point * a_points / (a_ms / 1e3) if a_ms > 0 else 0.0
+        scan_ceiling_ops = sm_count * SCAN_CEILING_POINTS_PER_CLK_SM * ops_per_point * \
+            float(peaks.get("sm_max_mhz", 1965.0)) * 1e6
         traffic = None
         prof = os.path.join(ROOT, "profiles", "k_eval_traffic.json")
         if os.path.exists(prof):
@@ -430,26 +503,36 @@ def main():
         clk = clocks.summary()
         cpu = None
         if world == 1 and not args.no_cpu_baseline:
-            cpu = cpu_baseline(desc, n_canon)
+            cpu = cpu_baseline(desc, n_canon, args.workload)
         line = {
             "metric": METRIC, "value": n_canon / (ms / 1e3), "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-            "config": {"workload": args.workload, "description": WORKLOADS[args.workload],
-                       "n_canon": n_canon, "survivors": survivors,
-                       "l2": "flushed between timed steps (256 MiB write)", "parallelism": "dp%d" % world,
-                       "gather": args.gather if world > 1 else None},
+            "config": config_dict(args, n_canon, survivors),
+            "l2": "flushed between timed steps (256 MiB write, outside the timed events)",
             "survivors_per_s": survivors / (ms / 1e3),
+            "gathered": {"ms_per_step": ms, "value": n_canon / (ms / 1e3)} if world > 1 else None,
+            "sharded_resident": sharded,
+            "count": count_line,
+            "replicas": {"l4_digests": ["0x%016x" % d for d in replicas], "ranks_agree": len(set(replicas)) == 1,
+                         "how": "digest of each rank's redundantly computed L1-L4 list, all-gathered"},
             "roofline": {"bound": "alu", "kernel": "k_eval<A> (L8-L9 A-read grids)",
                          "achieved": achieved / 1e12, "peak": peak_ops / 1e12, "unit": "T int16-ops/s",
                          "frac": achieved / peak_ops if peak_ops else None, "traffic": traffic,
+                         "peak_measured_scan": scan_ceiling_ops / 1e12,
+                         "frac_measured_scan": achieved / scan_ceiling_ops,
+                         "peak_measured_scan_source": "profiles/r02_micro: best packed-scan body %.2f points/clk/SM "
+                                                      "(scripts/micro/scan.cu) x SMs x sm_max_mhz x 2 ops"
+                                                      % SCAN_CEILING_POINTS_PER_CLK_SM,
                          "algorithmic_ops_per_launch": ops_per_point * a_points,
                          "avg_launch_ms": a_ms,
                          "peak_source": "%d SMs x %d int lane-instr/clk x 2 (16-bit halves) x sm_max_mhz (%s "
                                         "MEASURED_PEAKS.json); 2 int ops per point" % (sm_count, lanes, peak_src),
                          "points_per_s_kernel": a_points / (a_ms / 1e3) if a_ms > 0 else None},
             "e2e": {"value": n_canon / (e2e_step / 1e3), "unit": UNIT,
-                    "h2d_bytes_per_step": 96,
+                    "h2d_bytes_per_step": 0,
+                    "inputs": "a 96-byte space description, resolved into kernel parameters when the handle "
+                              "captures its pass; a replayed pass reads no host input",
                     "d2h_bytes_per_step": 16 * st_local["survivors"] + 512,
                     "ms_per_step": e2e_step,
                     "d2h_copy_ms": d2h_copy_ms,
@@ -565,53 +648,124 @@ def ir_measure(beast, desc, stream, flush, canonical_ms, reps=3):
 
 
 def _cpu_model():
+    """lscpu's model fields plus the microarchitecture they name (Intel
+    family 6 model numbers)."""
+    info = {}
     try:
-        for line in open("/proc/cpuinfo"):
-            if line.startswith("model name"):
-                return line.split(":", 1)[1].strip()
-    except OSError:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            k, _, v = line.partition(":")
+            info[k.strip()] = v.strip()
+    except Exception:
         pass
-    return None
+    if not info:
+        try:
+            for line in open("/proc/cpuinfo"):
+                k, _, v = line.partition(":")
+                k = {"model name": "Model name", "cpu family": "CPU family", "model": "Model",
+                     "stepping": "Stepping"}.get(k.strip())
+                if k and k not in info:
+                    info[k] = v.strip()
+        except OSError:
+            pass
+    uarch = {("6", "143"): "Sapphire Rapids", ("6", "207"): "Emerald Rapids", ("6", "173"): "Granite Rapids",
+             ("6", "106"): "Ice Lake-SP", ("6", "85"): "Skylake/Cascade Lake-SP"}.get(
+        (info.get("CPU family"), info.get("Model")))
+    return {"model_name": info.get("Model name"), "family": info.get("CPU family"), "model": info.get("Model"),
+            "stepping": info.get("Stepping"), "microarchitecture": uarch,
+            "sockets": info.get("Socket(s)"), "cores_per_socket": info.get("Core(s) per socket"),
+            "threads_per_core": info.get("Thread(s) per core")}
 
 
-def cpu_baseline(desc, n_canon=None, budget_s=10.0):
-    """The oracle nest on this host (SURVEY §8(d) "oracle timing beside it"):
-    all cores (OpenMP over dim_m; the reported value) and one thread.  Bounded
-    for the one-thread rate: the whole space if it takes at most budget_s,
-    else the canonical prefix dim_m <= D with D doubled from 1 while a run
-    stays under budget_s (the work is far from uniform in dim_m, so D is
-    found by measurement)."""
+def _oracle_run(desc, threads, budget_s):
+    """Oracle nest on `desc` with `threads` OpenMP threads: the whole space if
+    it takes at most budget_s, else the canonical prefix dim_m <= D with D
+    doubled from 1 while a run stays under budget_s (the work is far from
+    uniform in dim_m, so D is found by measurement).  Returns (D or None for
+    the whole space, points, survivors, seconds)."""
     import oracle
-    cores = os.cpu_count() or 1
     dmx = oracle.resolve(desc)["dim_m_max"]
+    d, best = 1, None
+    if threads > 1:
+        d = dmx                      # OpenMP is over dim_m: a prefix would starve the cores
+    while True:
+        dd = min(d, dmx)
+        t = time.perf_counter()
+        r = oracle.nest(desc if dd >= dmx else dict(desc, dim_m_max=dd), threads=threads, digest=False)
+        dt = time.perf_counter() - t
+        best = (None if dd >= dmx else dd, sum(r["visits"]), r["survivors"], dt)
+        if dd >= dmx or dt * 2.5 > budget_s:   # the next doubling would overrun the budget
+            return best
+        d *= 2
 
-    def run(threads):
-        d, best = 1, None
-        while True:
-            dd = min(d, dmx)
-            t = time.perf_counter()
-            r = oracle.nest(desc if dd >= dmx else dict(desc, dim_m_max=dd), threads=threads, digest=False)
-            dt = time.perf_counter() - t
-            best = (dd, r, dt)
-            if dd >= dmx or dt * 2.5 > budget_s:   # the next doubling would overrun the budget
-                return best
-            d *= 2
 
-    # all cores: the whole space (the OpenMP loop is over dim_m, so a dim_m
-    # prefix would starve the cores; the headline takes ~0.5 s, the largest
-    # configuration ~70 s); one thread: the doubling prefix
-    t = time.perf_counter()
-    r = oracle.nest(desc, threads=cores, digest=False)
-    d, dt = dmx, time.perf_counter() - t
-    d1, r1, dt1 = run(1)
-    pts = sum(r["visits"])
-    what = "whole space once" if d >= dmx else "canonical prefix dim_m <= %d of the space" % d
+def cpu_baseline(desc, n_canon=None, workload="headline", budget_s=10.0):
+    """The oracle nest on this host (SURVEY §8(d) "oracle timing beside it"):
+    the bench workload on all cores (the reported value; whole space) and on
+    one thread (bounded prefix), plus both rates over BASELINE configs[0..2]
+    (tiny DGEMM; the headline; SGEMM, CGEMM, ZGEMM x 4 transposes with K40c
+    limits), with the host CPU model; N_space (the unpruned space, closed
+    form) as context."""
+    import beast_inputs as bi
+    import oracle.closed_form
+    cores = os.cpu_count() or 1
+    d_all, pts, surv, dt = _oracle_run(desc, cores, 1e9)
+    d1, pts1, _, dt1 = _oracle_run(desc, 1, budget_s)
+    configs = []
+    groups = [("configs[0] tiny DGEMM NN", [bi.tiny("D")]),
+              ("configs[1] headline DGEMM NN K40c", [bi.headline()]),
+              ("configs[2] S/C/Z x 4 transposes K40c",
+               [bi.k40c(p, a, b) for p in ("S", "C", "Z") for a, b in bi.TRANSPOSES])]
+    for name, spaces in groups:
+        tot_p = tot_s = tot_t = 0.0
+        for sp in spaces:
+            _, p_, s_, t_ = _oracle_run(sp, cores, 1e9)
+            tot_p += p_
+            tot_s += s_
+            tot_t += t_
+        # one thread: the first space of the group, bounded
+        dd, p1, _, t1 = _oracle_run(spaces[0], 1, budget_s / 2)
+        configs.append({"config": name, "spaces": len(spaces), "points": int(tot_p), "survivors": int(tot_s),
+                        "all_cores": {"s": tot_t, "points_per_s": tot_p / tot_t, "survivors_per_s": tot_s / tot_t},
+                        "single_thread": {"s": t1, "points_per_s": p1 / t1,
+                                          "sample": "whole first space" if dd is None else
+                                          "first space, canonical prefix dim_m <= %d" % dd}})
     return {"value": pts / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
-            "sample": "%s (%d points, %.1f s wall on %d threads), canonical nest" % (what, pts, dt, cores),
-            "survivors_per_s": r["survivors"] / dt,
-            "single_thread": {"value": sum(r1["visits"]) / dt1, "unit": UNIT, "s": dt1,
-                              "sample": "whole space" if d1 >= dmx else "canonical prefix dim_m <= %d" % d1},
-            "cpu": _cpu_model()}
+            "sample": "whole %s space once (%d points, %.1f s wall on %d threads), canonical nest"
+                      % (workload, pts, dt, cores),
+            "survivors_per_s": surv / dt,
+            "single_thread": {"value": pts1 / dt1, "unit": UNIT, "s": dt1,
+                              "sample": "whole space" if d1 is None else "canonical prefix dim_m <= %d" % d1},
+            "configs": configs, "cpu": _cpu_model(),
+            "n_space": str(oracle.closed_form.n_space(desc)),
+            "n_space_note": "size of the unpruned dependent-range space (closed form, context only; never a rate)"}
+
+
+def relaunch(args):
+    """`--gpus N` (N > 1) without a launcher: start N ranks on this node
+    under torch.distributed.run (127.0.0.1) with this command line; rank 0
+    prints the JSON line.  Fails (exit 2) if fewer than N GPUs are visible."""
+    import socket
+    try:
+        import torch
+        visible = torch.cuda.device_count()
+    except Exception:
+        visible = 0
+    if visible < args.gpus:
+        print("bench.py: --gpus %d but only %d CUDA device(s) visible; not measuring" % (args.gpus, visible),
+              file=sys.stderr)
+        return 2
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")              # communicator / transport lines (NVLS, P2P) ...
+    env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    env.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")  # ... on stderr, so stdout carries only the JSON line
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", str(args.gpus),
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd, env=env)
 
 
 if __name__ == "__main__":

@@ -26,8 +26,12 @@
  *   - A beast_space handle owns its device scratch (allocated on first use,
  *     grown on demand, kept until beast_space_destroy) through the allocator
  *     set with beast_space_set_allocator (default cudaMalloc / cudaFree).  A
- *     handle is not safe for concurrent calls; separate handles are
- *     independent.  Device calls run on the CUDA device current at call
+ *     handle is not safe for concurrent calls from several host threads;
+ *     separate handles are independent.  The passes of one handle share its
+ *     scratch, so a pass enqueued on a stream other than the previous pass's
+ *     first waits (cudaStreamWaitEvent) for the end of that pass;
+ *     beast_space_destroy waits for the handle's last pass before releasing
+ *     the scratch.  Device calls run on the CUDA device current at call
  *     time, which must not change over the handle's life.
  *   - rank / world select a shard: the contiguous canonical range of L4
  *     survivors (dim_m, dim_n, blk_m, blk_n) whose cumulative estimated
@@ -50,7 +54,7 @@
 extern "C" {
 #endif
 
-#define BEAST_ABI_VERSION 1
+#define BEAST_ABI_VERSION 2
 
 typedef enum {
     BEAST_OK = 0,
@@ -120,7 +124,21 @@ typedef struct {
  *   11 cant_reshape_b2
  * Levels L1..L6 and predicates 0..7 are charged to rank 0 only (every rank
  * recomputes them); summing the stats of all ranks gives the whole space.
- * points_evaluated = sum(visits). */
+ * points_evaluated = sum(visits).
+ *
+ * Evaluation evidence (SURVEY §8(d) honesty rule: the instrumented run shows
+ * what the timed run evaluates).  The A-read (L8-L9) and B-read (L10-L11)
+ * grids of a job are evaluated row by row -- a row holds the short-axis
+ * coordinate fixed and runs the long one over 1..L -- by a packed scan that
+ * forms 16 points per loop iteration.  formed[s] (s = 0: A grids, 1: B
+ * grids) counts 16 per executed iteration of every live row, counted inside
+ * the scan loop, so formed[0] = sum over rows of 16 * ceil(L / 16) >=
+ * visits[8] (the excess is each row's padding to whole 16-point blocks) and
+ * likewise formed[1] >= visits[10].  checked[s]: rows whose scan found a
+ * candidate zero and were then checked exactly (>= the a1 / b1 passes).
+ * l4_digest: order-sensitive digest sum_i sm64(w_i ^ sm64(i)) of this call's
+ * list of L4 survivors (levels L1-L4, computed redundantly by every rank:
+ * equal on every rank of one space; sm64 as in beast_digest). */
 typedef struct {
     uint64_t visits[15];
     uint64_t rejected[12];
@@ -128,6 +146,9 @@ typedef struct {
     uint64_t prefixes;          /* L7 prefixes in this shard */
     uint64_t valid_a;           /* (prefix, dim_m_a, dim_n_a) passing a1 and a2 */
     uint64_t tuples;            /* (prefix, A grid, B grid) survivors; survivors = 16 * tuples */
+    uint64_t formed[2];         /* points formed by the packed scan, A / B grids (stats runs only) */
+    uint64_t checked[2];        /* rows checked exactly, A / B grids (stats runs only) */
+    uint64_t l4_digest;         /* digest of the L4 survivor list (every run) */
 } beast_stats;
 
 /* One surviving variant, 16 bytes, 16-byte aligned; as a little-endian
@@ -251,7 +272,8 @@ int beast_enumerate_to_host_async(beast_space *space, int rank, int world, void 
 /* Wait for the most recent pass of the handle (synchronous or asynchronous)
  * to complete -- and, after beast_enumerate_to_host_async, its host copy;
  * *written: host, out, the records of that pass.  BEAST_ERR_CAPACITY if they
- * exceeded the capacity of the last asynchronous call; BEAST_ERR_WORKSPACE if
+ * exceeded the capacity of that pass's record buffer (counting passes have
+ * none); BEAST_ERR_WORKSPACE if
  * an asynchronous pass overflowed its scratch or a host pass's count differed
  * from the copied one. */
 int beast_wait(beast_space *space, void *stream, uint64_t *written);
@@ -400,6 +422,13 @@ int beast_last_launches(const beast_space *space, uint64_t *kernels, float *a_ev
  * beast_enumerate_to_host on this handle; -1 if that call wrote no list or
  * timing was off.  *ms: host, out. */
 int beast_last_write_ms(const beast_space *space, float *ms);
+
+/* beast_stats.l4_digest of the last completed pass on this handle (any mode,
+ * stats or not): the digest of its L4 survivor list, which every rank of a
+ * sharded run computes redundantly -- the multi-GPU combine all-gathers it
+ * and checks that the ranks agree.  *digest: host, out.
+ * BEAST_ERR_INVALID_ARGUMENT before the first pass. */
+int beast_last_l4_digest(const beast_space *space, uint64_t *digest);
 
 #ifdef __cplusplus
 }

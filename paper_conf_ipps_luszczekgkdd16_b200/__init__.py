@@ -209,7 +209,8 @@ def stats_dict(st: beast_stats) -> dict:
     return dict(visits=[int(x) for x in st.visits], rejected=[int(x) for x in st.rejected],
                 survivors=int(st.survivors), prefixes=int(st.prefixes),
                 valid_a=int(st.valid_a), tuples=int(st.tuples),
-                points=int(sum(st.visits)))
+                formed=[int(x) for x in st.formed], checked=[int(x) for x in st.checked],
+                l4_digest=int(st.l4_digest), points=int(sum(st.visits)))
 
 
 # ----------------------------------------------------------- convenience
@@ -305,6 +306,12 @@ class Space:
         ms = ctypes.c_float(0)
         _check(_lib.lib().beast_last_write_ms(self.handle, ctypes.byref(ms)))
         return float(ms.value)
+
+    def last_l4_digest(self):
+        """Digest of the L4 survivor list of the last pass (beast_last_l4_digest)."""
+        d = ctypes.c_uint64(0)
+        _check(_lib.lib().beast_last_l4_digest(self.handle, ctypes.byref(d)), self.handle)
+        return int(d.value)
 
     def close(self):
         if self.handle:

@@ -55,7 +55,9 @@ class beast_bounds(ctypes.Structure):
 class beast_stats(ctypes.Structure):
     _fields_ = [("visits", ctypes.c_uint64 * 15), ("rejected", ctypes.c_uint64 * 12),
                 ("survivors", ctypes.c_uint64), ("prefixes", ctypes.c_uint64),
-                ("valid_a", ctypes.c_uint64), ("tuples", ctypes.c_uint64)]
+                ("valid_a", ctypes.c_uint64), ("tuples", ctypes.c_uint64),
+                ("formed", ctypes.c_uint64 * 2), ("checked", ctypes.c_uint64 * 2),
+                ("l4_digest", ctypes.c_uint64)]
 
 
 _cpp = ctypes.POINTER(ctypes.c_char_p)
@@ -115,6 +117,7 @@ _sig = {
     "beast_last_stage_ms": ([_vp, _P(ctypes.c_float)], ctypes.c_int),
     "beast_last_launches": ([_vp, _u64p, _P(ctypes.c_float), _u64p], ctypes.c_int),
     "beast_last_write_ms": ([_vp, ctypes.POINTER(ctypes.c_float)], ctypes.c_int),
+    "beast_last_l4_digest": ([_vp, _u64p], ctypes.c_int),
 }
 for _name, (_args, _res) in _sig.items():
     _f = getattr(_L, _name)

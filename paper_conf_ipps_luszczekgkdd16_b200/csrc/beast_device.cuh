@@ -82,6 +82,14 @@ __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
 
 __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31; }
 
+// splitmix64 finaliser (the digests of include/beast.h)
+__device__ __forceinline__ uint64_t sm64(uint64_t z) {
+    z += 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
 __device__ __forceinline__ uint64_t ld_volatile_u64(const uint64_t *p) {
     uint64_t v;
     asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(v) : "l"(p));
@@ -214,7 +222,11 @@ __device__ __forceinline__ uint32_t vmin_u16x2(uint32_t a, uint32_t b) {
 // products past L are computed but a match there is rejected by the exact
 // check (t <= L).  Returns the running per-half minimum: a zero half marks a
 // candidate row.
-__device__ __forceinline__ uint32_t scan_rows(uint32_t s1, uint32_t s2, uint32_t T, uint32_t NB) {
+// COUNT (instrumented build): *blocks is incremented inside the loop body,
+// once per executed 16-point iteration (beast_stats.formed).
+template <bool COUNT = false>
+__device__ __forceinline__ uint32_t scan_rows(uint32_t s1, uint32_t s2, uint32_t T, uint32_t NB,
+                                              uint32_t *blocks = nullptr) {
     const uint32_t Sp = s1 | (s2 << 16);
     uint32_t Cb = (0x10000u - T) * 0x10001u;
     asm volatile("" : "+r"(Cb));             // keep C as one register (no per-block re-derivation)
@@ -228,6 +240,7 @@ __device__ __forceinline__ uint32_t scan_rows(uint32_t s1, uint32_t s2, uint32_t
     for (uint32_t b = 0; b < NB; ++b) {
         eval16pp<KI>(acc, acc2, Cb, Sp, M);
         Cb += step;
+        if (COUNT) ++*blocks;
     }
     return vmin_u16x2(acc, acc2);
 }

@@ -21,7 +21,11 @@ from __future__ import annotations
 import torch
 import torch.distributed as dist
 
-STAT_LEN = 15 + 12 + 4   # visits, rejected, survivors, prefixes, valid_a, tuples
+STAT_LEN = 15 + 12 + 4 + 4   # visits, rejected, survivors, prefixes, valid_a, tuples, formed[2], checked[2]
+
+
+class ReplicaMismatch(RuntimeError):
+    """The ranks' redundantly computed L1-L4 lists differ."""
 
 
 def _dev():
@@ -31,26 +35,56 @@ def _dev():
 
 def stats_to_tensor(st: dict, device=None) -> torch.Tensor:
     v = list(st["visits"]) + list(st["rejected"]) + [st["survivors"], st["prefixes"], st["valid_a"], st["tuples"]]
+    v += list(st.get("formed", (0, 0))) + list(st.get("checked", (0, 0)))
     return torch.tensor(v, dtype=torch.int64, device=device or _dev())
 
 
 def tensor_to_stats(t: torch.Tensor) -> dict:
     v = [int(x) for x in t.cpu().tolist()]
-    st = dict(visits=v[:15], rejected=v[15:27], survivors=v[27], prefixes=v[28], valid_a=v[29], tuples=v[30])
+    st = dict(visits=v[:15], rejected=v[15:27], survivors=v[27], prefixes=v[28], valid_a=v[29], tuples=v[30],
+              formed=v[31:33], checked=v[33:35])
     st["points"] = sum(st["visits"])
     return st
 
 
+def _u64_to_i64(x: int) -> int:
+    return x - (1 << 64) if x >= (1 << 63) else x
+
+
+def check_replicas(l4_digest: int, world: int, device=None) -> list:
+    """every rank computes levels L1-L4 redundantly; all-gather
+    the 64-bit digest of each rank's L4 survivor list (beast_stats.l4_digest
+    / Space.last_l4_digest) and raise ReplicaMismatch unless all ranks
+    agree.  Returns the gathered digests (unsigned)."""
+    if world <= 1 or not dist.is_initialized():
+        return [int(l4_digest)]
+    dev = device or _dev()
+    mine = torch.tensor([_u64_to_i64(int(l4_digest))], dtype=torch.int64, device=dev)
+    allv = [torch.zeros(1, dtype=torch.int64, device=dev) for _ in range(world)]
+    dist.all_gather(allv, mine)
+    got = [int(x.item()) & ((1 << 64) - 1) for x in allv]
+    if len(set(got)) != 1:
+        raise ReplicaMismatch("L4 survivor lists differ across ranks: digests %s" % ["0x%016x" % d for d in got])
+    return got
+
+
 def combine_stats(st: dict, world: int) -> dict:
     """Sum the per-shard statistics over all ranks (each level L1..L6 is
-    charged to rank 0 only by the library, so the sum is the whole space)."""
+    charged to rank 0 only by the library, so the sum is the whole space);
+    the L4 digest is checked equal across ranks (check_replicas) instead of
+    summed."""
     if world <= 1 or not dist.is_initialized():
         out = dict(st)
         out["points"] = sum(st["visits"])
         return out
+    if "l4_digest" in st:
+        check_replicas(st["l4_digest"], world)
     t = stats_to_tensor(st)
     dist.all_reduce(t, op=dist.ReduceOp.SUM)
-    return tensor_to_stats(t)
+    out = tensor_to_stats(t)
+    if "l4_digest" in st:
+        out["l4_digest"] = st["l4_digest"]
+    return out
 
 
 def shard_offsets(n_local: int, world: int, device=None) -> list:
@@ -157,14 +191,26 @@ class FusedGather:
     def run(self, space, stream=None) -> int:
         """One fused enumeration + gather; returns the global record count.
         On rank 0, self.buf[:total] then holds the canonical list (int64 view
-        of the (lo, hi) records)."""
+        of the (lo, hi) records).
+
+        Order: stage (local) -> all-gather of the counts -> every rank checks
+        the total against the capacity (the same counts everywhere, so all
+        ranks raise together and none is left waiting in a barrier) ->
+        barrier (rank 0 has finished with the previous list before any rank
+        overwrites it) -> write into rank 0's buffer -> barrier (the list is
+        complete)."""
         from . import beast_enumerate_stage, beast_write_at
         beast_enumerate_stage(space.handle, self.d_count, self.rank, self.world, stream)
         if self.world > 1:
             dist.all_gather_into_tensor(self.d_counts, self.d_count, group=self.group)
         else:
             self.d_counts.copy_(self.d_count)
+        total = int(self.d_counts.sum().item())
+        if total > self.capacity:
+            raise ValueError("fused gather: %d records exceed the buffer's capacity %d" % (total, self.capacity))
+        if self.hdl is not None:
+            self.hdl.barrier()
         beast_write_at(space.handle, self.root_ptr, self.capacity, self.d_counts, self.rank, self.world, stream)
         if self.hdl is not None:
             self.hdl.barrier()
-        return int(self.d_counts.sum().item())
+        return total

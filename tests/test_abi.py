@@ -45,7 +45,12 @@ def test_binding_names_match_abi(beast):
 
 
 def test_abi_version(beast):
-    assert beast.beast_abi_version() == 1
+    import ctypes
+    import re
+    hdr = open(os.path.join(ROOT, "include", "beast.h")).read()
+    assert beast.beast_abi_version() == int(re.search(r"#define BEAST_ABI_VERSION (\d+)", hdr).group(1)) == 2
+    # beast_stats: 15 visits + 12 rejections + 4 counts + formed[2] + checked[2] + l4_digest
+    assert ctypes.sizeof(beast.beast_stats) == 8 * (15 + 12 + 4 + 2 + 2 + 1)
 
 
 def test_k40c_preset_is_fig8_and_fig9(beast):

@@ -50,6 +50,17 @@ def _worker(rank, world, port, q):
         assert tot["survivors"] == len(full)
         assert tot["visits"] == [sum(range(1, world + 1))] * 15
         assert tot["valid_a"] == world and tot["points"] == 15 * sum(range(1, world + 1))
+        # SURVEY §8(e) replica check: the L4 digests all-gathered; equal ->
+        # passes, one rank different -> every rank raises (no rank hangs)
+        st.update(l4_digest=0xFEDCBA9876543210, formed=[5, 6], checked=[1, 2])
+        tot = bdist.combine_stats(st, world)
+        assert tot["l4_digest"] == 0xFEDCBA9876543210 and tot["formed"] == [5 * world, 6 * world]
+        assert bdist.check_replicas(0x1234, world) == [0x1234] * world
+        try:
+            bdist.check_replicas(0x1234 + (rank == world - 1), world)
+            raise AssertionError("mismatch not detected")
+        except bdist.ReplicaMismatch:
+            pass
         q.put((rank, "ok"))
     except Exception as e:  # pragma: no cover - reported to the parent
         q.put((rank, repr(e)))

@@ -47,9 +47,32 @@ def test_bench_json_line_contract():
     assert d["gpu_launches"] > 0
     c = d["cpu_baseline"]
     assert c["kind"] == "oracle" and c["cores"] >= 1 and c["value"] > 0 and c["single_thread"]["value"] > 0
+    # count timed on its own, N_space as context, the oracle
+    # over configs[0..2] with the CPU model, the measured-scan fraction
+    assert d["count"]["value"] > 0 and d["count"]["ms_per_step"] > 0
+    assert [x["config"][:10] for x in c["configs"]] == ["configs[0]", "configs[1]", "configs[2]"]
+    assert c["configs"][1]["points"] == 2_096_997_743 and c["configs"][2]["spaces"] == 12
+    assert int(c["n_space"]) > d["config"]["n_canon"] and c["cpu"]["model_name"]
+    assert 0 < r["frac_measured_scan"] < r["frac"]
+    assert d["sharded_resident"] is None and d["replicas"]["ranks_agree"] is True
+    assert e["h2d_bytes_per_step"] == 0
 
 
 def test_bench_reference_arm():
     d = _run("--impl", "reference", "--workload", "widened256_k40c", "--steps", "3", "--warmup", "3")
     assert d["impl"] == "reference" and d["value"] > 0
     assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["cpu_baseline"]["kind"] == "oracle"
+    g = _run("--workload", "widened256_k40c", "--steps", "3", "--warmup", "3", "--no-sweep", "--no-ir",
+             "--no-cpu-baseline")
+    assert d["config"] == g["config"]                  # the driver's same-config check
+
+
+def test_bench_gpus_more_than_visible_fails_loudly():
+    """--gpus N without a launcher starts N ranks itself; with fewer GPUs than
+    N visible it must fail, not measure one GPU and print n_gpus 1."""
+    import torch
+    n = torch.cuda.device_count()
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", str(n + 1), "--steps", "3"],
+                         cwd=ROOT, capture_output=True, text=True, timeout=600)
+    assert out.returncode != 0 and "visible" in out.stderr
+    assert not [l for l in out.stdout.splitlines() if l.startswith("{")]

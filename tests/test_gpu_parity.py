@@ -11,11 +11,18 @@ from __future__ import annotations
 import os
 import random
 
+import json
+
 import numpy as np
 import pytest
 
 import beast_inputs as bi
 import oracle
+import oracle.analytic
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+with open(os.path.join(ROOT, "tests", "golden", "wide_fuzz.json")) as _f:
+    WIDE = json.load(_f)["spaces"]
 
 pytestmark = pytest.mark.gpu
 
@@ -44,6 +51,31 @@ def _run(beast, desc, rank=0, world=1, stats=True):
     return got, st, dig, n
 
 
+def _formed(shapes):
+    """Points the packed scan forms over grids of the given shape histogram
+    (include/beast.h, beast_stats.formed): a grid of m x n points is
+    min(m, n) rows of max(m, n) points, each row run in whole 16-point
+    blocks."""
+    tot = 0
+    for (m, n), c in shapes.items():
+        tot += c * min(m, n) * 16 * ((max(m, n) + 15) // 16)
+    return tot
+
+
+def _check_evaluated(desc, st, exact=True):
+    """The instrumented run formed every canonical A and B grid point (and
+    only the row padding on top): formed == the oracle's grid shapes in the
+    row layout (exact) or visits <= formed <= visits + 15 rows (bound)."""
+    v, rej = st["visits"], st["rejected"]
+    if exact:
+        sh = oracle.analytic.count(desc, shapes=True)
+        assert st["formed"] == [_formed(sh["a_shapes"]), _formed(sh["b_shapes"])]
+    assert v[8] <= st["formed"][0] <= v[8] + 15 * v[7]
+    assert v[10] <= st["formed"][1] <= v[10] + 15 * v[9]
+    # every row with a point passing a1 (b1) was checked exactly
+    assert st["checked"][0] >= v[8] - rej[8] and st["checked"][1] >= v[10] - rej[9]
+
+
 def _check_small(beast, desc):
     got, st, dig, n = _run(beast, desc)
     ref = oracle.nest(desc, records=True)
@@ -55,6 +87,7 @@ def _check_small(beast, desc):
     assert st["rejected"] == ref["rejected"], (st["rejected"], ref["rejected"])
     if len(got):
         assert dig == ref["digest"]
+    _check_evaluated(desc, st)
 
 
 @pytest.mark.parametrize("p", bi.PRECISIONS)
@@ -70,6 +103,25 @@ def test_micro(beast):
 @pytest.mark.parametrize("seed", range(200))
 def test_fuzz(beast, seed):
     _check_small(beast, bi.fuzz_space(seed))
+
+
+@pytest.mark.parametrize("seed", range(200, 400))
+def test_fuzz_wide(beast, seed):
+    """The library's whole admitted input range (beast_inputs.fuzz_space_wide:
+    threads_per_block up to 65535, float_size up to 1024, max_blocks up to
+    65534, thresholds up to 2^30 / 2^20, limits up to 2^31 - 1, bounds up to
+    4095), bit-exact against the oracle run here (and its fixture)."""
+    e = WIDE[str(seed)]
+    desc = bi.fuzz_space_wide(seed, e["attempt"])
+    assert desc == e["space"]
+    got, st, dig, n = _run(beast, desc)
+    assert n == st["survivors"] == e["survivors"]
+    assert st["visits"] == e["visits"] and st["rejected"] == e["rejected"]
+    if n:
+        assert "0x%016x" % dig == e["digest"]
+    ref = oracle.nest(desc, threads=os.cpu_count(), records=True)
+    assert np.array_equal(got, _oracle_lohi(ref["records"]))
+    _check_evaluated(desc, st, exact=e["n_canon"] < 50_000_000)
 
 
 def test_empty_space(beast):
@@ -92,13 +144,15 @@ def test_headline_bit_exact(beast):
     assert np.array_equal(got, _oracle_lohi(ref["records"]))
     assert st["visits"] == ref["visits"] and st["rejected"] == ref["rejected"]
     assert dig == ref["digest"] and n == 1_207_600
+    _check_evaluated(desc, st)
 
 
 GOLDEN_BIG = ["k40c_%s_%d%d" % (p, a, b) for p in bi.PRECISIONS for a, b in bi.TRANSPOSES] + \
              ["b200_%s_%d%d" % (p, a, b) for p in bi.PRECISIONS for a, b in bi.TRANSPOSES] + \
              ["widened%d_%s_D_00" % (w, d) for w in (64, 256, 512) for d in ("k40c", "b200")] + \
              ["b200_48k_D_00", "b200_48k_S_00"] + \
-             ["maxbound_k40c_D_00", "maxbound_k40c_Z_11", "maxbound_b200_D_00"]
+             ["maxbound_k40c_D_00", "maxbound_k40c_Z_11", "maxbound_b200_D_00"] + \
+             sorted(bi.EXTREME)
 
 
 @pytest.mark.parametrize("key", GOLDEN_BIG)
@@ -113,6 +167,7 @@ def test_full_size_vs_golden(beast, golden_expected, key):
         assert st["visits"] == e["visits"], key
         assert st["rejected"] == e["rejected"], key
         assert "0x%016x" % beast.beast_digest(rec) == e["digest"], key
+        _check_evaluated(e["space"], st, exact=False)
         if e["first"]:
             lo, hi = rec[0].cpu().numpy(), rec[-1].cpu().numpy()
             assert ["%016x" % lo[1], "%016x" % lo[0]] == e["first"]
