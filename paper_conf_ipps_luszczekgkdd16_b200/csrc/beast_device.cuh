@@ -182,7 +182,7 @@ __device__ __forceinline__ uint64_t cta_exclusive_scan64(uint64_t v, uint64_t *s
 #define BEAST_SCAN_KI 12
 #endif
 #ifndef BEAST_SCAN_UNROLL
-#define BEAST_SCAN_UNROLL 2
+#define BEAST_SCAN_UNROLL 4
 #endif
 #define BEAST_PRAGMA(x) _Pragma(#x)
 #define BEAST_UNROLL(n) BEAST_PRAGMA(unroll n)
@@ -222,11 +222,7 @@ __device__ __forceinline__ uint32_t vmin_u16x2(uint32_t a, uint32_t b) {
 // products past L are computed but a match there is rejected by the exact
 // check (t <= L).  Returns the running per-half minimum: a zero half marks a
 // candidate row.
-// COUNT (instrumented build): *blocks is incremented inside the loop body,
-// once per executed 16-point iteration (beast_stats.formed).
-template <bool COUNT = false>
-__device__ __forceinline__ uint32_t scan_rows(uint32_t s1, uint32_t s2, uint32_t T, uint32_t NB,
-                                              uint32_t *blocks = nullptr) {
+__device__ __forceinline__ uint32_t scan_rows(uint32_t s1, uint32_t s2, uint32_t T, uint32_t NB) {
     const uint32_t Sp = s1 | (s2 << 16);
     uint32_t Cb = (0x10000u - T) * 0x10001u;
     asm volatile("" : "+r"(Cb));             // keep C as one register (no per-block re-derivation)
@@ -240,7 +236,29 @@ __device__ __forceinline__ uint32_t scan_rows(uint32_t s1, uint32_t s2, uint32_t
     for (uint32_t b = 0; b < NB; ++b) {
         eval16pp<KI>(acc, acc2, Cb, Sp, M);
         Cb += step;
-        if (COUNT) ++*blocks;
+    }
+    return vmin_u16x2(acc, acc2);
+}
+
+// The same scan in the instrumented build: `blocks` is incremented inside
+// the loop body, once per executed 16-point iteration (beast_stats.formed).
+// (A separate function, so the timed kernels keep scan_rows' exact code.)
+__device__ __forceinline__ uint32_t scan_rows_counted(uint32_t s1, uint32_t s2, uint32_t T, uint32_t NB,
+                                                      uint32_t &blocks) {
+    const uint32_t Sp = s1 | (s2 << 16);
+    uint32_t Cb = (0x10000u - T) * 0x10001u;
+    asm volatile("" : "+r"(Cb));
+    const uint32_t step = Sp << 4;
+    constexpr int KI = BEAST_SCAN_KI;
+    uint32_t M[16 - KI + (KI == 16)];
+#pragma unroll
+    for (int i = 0; i < 16 - KI; ++i) M[i] = Sp * (uint32_t)(KI + 1 + i);
+    uint32_t acc = 0xffffffffu, acc2 = 0xffffffffu;
+    BEAST_UNROLL(BEAST_SCAN_UNROLL)
+    for (uint32_t b = 0; b < NB; ++b) {
+        eval16pp<KI>(acc, acc2, Cb, Sp, M);
+        Cb += step;
+        asm volatile("add.u32 %0, %0, 1;" : "+r"(blocks));   // counted where the block runs
     }
     return vmin_u16x2(acc, acc2);
 }
