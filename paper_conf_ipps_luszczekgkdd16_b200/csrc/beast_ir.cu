@@ -189,6 +189,7 @@ struct beast_ir {
     std::vector<cudaKernel_t> k_count, k_emit;     // per level, warp per parent
     std::vector<cudaKernel_t> k_tcount, k_temit;   // per level, thread per parent
     std::vector<cudaKernel_t> k_fcount, k_femit;   // levels k and k + 1 fused (k without constraints), else null
+    std::vector<cudaKernel_t> k_wfcount, k_wfemit; // the same, warp per parent
     cudaKernel_t k_root = nullptr, k_tiles = nullptr, k_top = nullptr,
                  k_add = nullptr;
     int sm_count = 148;
@@ -311,6 +312,19 @@ std::string generate(const beast_ir *ir) {
                      ir->dnames[d] + ";\n";
         return c;
     };
+    // first-failing counters of a level's nck constraints: registers (a
+    // dynamically indexed array would live in local memory)
+    auto rej_decl = [&](int nck) {
+        std::string c = "";
+        for (int l = 0; l < nck; ++l) c += "    u64 ir_rej" + std::to_string(l) + "_ = 0;\n";
+        return c;
+    };
+    auto rej_inc = [&](int nck, const char *ind) {
+        std::string c = std::string(ind) + "if (ir_r_ == 0) ++ir_c_;\n";
+        for (int l = 0; l < nck; ++l)
+            c += std::string(ind) + "else if (ir_r_ == " + std::to_string(l + 1) + ") ++ir_rej" + std::to_string(l) + "_;\n";
+        return c;
+    };
     auto constraints_at = [&](int k, const char *ind, std::vector<int> *idx) {
         std::string c;
         int local = 0;
@@ -363,20 +377,18 @@ std::string generate(const beast_ir *ir) {
                  "u64 *ir_cnt_, u64 *ir_stats_) {\n", k);
         s += buf;
         s += head + consts;
-        snprintf(buf, sizeof(buf), "    u64 ir_vis_ = 0, ir_rej_[%d];\n    for (int ir_q_ = 0; ir_q_ < %d; ++ir_q_) ir_rej_[ir_q_] = 0;\n",
-                 nck > 0 ? nck : 1, nck);
-        s += buf;
+        s += "    u64 ir_vis_ = 0;\n" + rej_decl(nck);
         s += "    for (u64 ir_p_ = ir_w0_; ir_p_ < ir_npar_; ir_p_ += ir_nw_) {\n" + parent;
         s += "        ir_vis_ += ir_n_;\n        u64 ir_c_ = 0;\n";
         s += "        for (u64 ir_i_ = ir_lane_; ir_i_ < ir_n_; ir_i_ += 32) {\n" + point;
-        if (nck) s += "            if (ir_r_ == 0) ++ir_c_; else ir_rej_[ir_r_ - 1] += 1;\n";
+        if (nck) s += rej_inc(nck, "            ");
         else s += "            ++ir_c_;\n";
         s += "        }\n        ir_c_ = warp_sum(ir_c_);\n        if (ir_lane_ == 0) ir_cnt_[ir_p_] = ir_c_;\n    }\n";
         snprintf(buf, sizeof(buf), "    if (ir_lane_ == 0 && ir_vis_) atomicAdd(&ir_stats_[%d], ir_vis_);\n", k);
         s += buf;
         for (int l = 0; l < nck; ++l) {
             snprintf(buf, sizeof(buf),
-                     "    { const u64 ir_x_ = warp_sum(ir_rej_[%d]); if (ir_lane_ == 0 && ir_x_) atomicAdd(&ir_stats_[NI + %d], ir_x_); }\n",
+                     "    { const u64 ir_x_ = warp_sum(ir_rej%d_); if (ir_lane_ == 0 && ir_x_) atomicAdd(&ir_stats_[NI + %d], ir_x_); }\n",
                      l, idx[l]);
             s += buf;
         }
@@ -418,20 +430,18 @@ std::string generate(const beast_ir *ir) {
                  "u64 *ir_cnt_, u64 *ir_stats_) {\n", k);
         s += buf;
         s += thead + consts;
-        snprintf(buf, sizeof(buf), "    u64 ir_vis_ = 0, ir_rej_[%d];\n    for (int ir_q_ = 0; ir_q_ < %d; ++ir_q_) ir_rej_[ir_q_] = 0;\n",
-                 nck > 0 ? nck : 1, nck);
-        s += buf;
+        s += "    u64 ir_vis_ = 0;\n" + rej_decl(nck);
         s += "    for (u64 ir_p_ = ir_t0_; ir_p_ < ir_npar_; ir_p_ += ir_nt_) {\n" + parent;
         s += "        ir_vis_ += ir_n_;\n        u64 ir_c_ = 0;\n";
         s += "        for (u64 ir_i_ = 0; ir_i_ < ir_n_; ++ir_i_) {\n" + point;
-        if (nck) s += "            if (ir_r_ == 0) ++ir_c_; else ir_rej_[ir_r_ - 1] += 1;\n";
+        if (nck) s += rej_inc(nck, "            ");
         else s += "            ++ir_c_;\n";
         s += "        }\n        ir_cnt_[ir_p_] = ir_c_;\n    }\n";
         snprintf(buf, sizeof(buf), "    ir_vis_ = warp_sum(ir_vis_);\n    if (ir_lane_ == 0 && ir_vis_) atomicAdd(&ir_stats_[%d], ir_vis_);\n", k);
         s += buf;
         for (int l = 0; l < nck; ++l) {
             snprintf(buf, sizeof(buf),
-                     "    { const u64 ir_x_ = warp_sum(ir_rej_[%d]); if (ir_lane_ == 0 && ir_x_) atomicAdd(&ir_stats_[NI + %d], ir_x_); }\n",
+                     "    { const u64 ir_x_ = warp_sum(ir_rej%d_); if (ir_lane_ == 0 && ir_x_) atomicAdd(&ir_stats_[NI + %d], ir_x_); }\n",
                      l, idx[l]);
             s += buf;
         }
@@ -498,16 +508,13 @@ std::string generate(const beast_ir *ir) {
                  "u64 *ir_cnt_, u64 *ir_stats_) {\n", k);
         s += buf;
         s += thead + consts;
-        snprintf(buf, sizeof(buf),
-                 "    u64 ir_vis_ = 0, ir_vis2_ = 0, ir_rej_[%d];\n    for (int ir_q_ = 0; ir_q_ < %d; ++ir_q_) ir_rej_[ir_q_] = 0;\n",
-                 nck > 0 ? nck : 1, nck);
-        s += buf;
+        s += "    u64 ir_vis_ = 0, ir_vis2_ = 0;\n" + rej_decl(nck);
         s += "    for (u64 ir_p_ = ir_t0_; ir_p_ < ir_npar_; ir_p_ += ir_nt_) {\n" + parent;
         s += "        ir_vis_ += ir_n_;\n        u64 ir_c_ = 0;\n";
         s += "        for (u64 ir_i_ = 0; ir_i_ < ir_n_; ++ir_i_) {\n" + outer;
         s += "            ir_vis2_ += ir_n2_;\n";
         s += "            for (u64 ir_j_ = 0; ir_j_ < ir_n2_; ++ir_j_) {\n" + inner;
-        if (nck) s += "                if (ir_r_ == 0) ++ir_c_; else ir_rej_[ir_r_ - 1] += 1;\n";
+        if (nck) s += rej_inc(nck, "                ");
         else s += "                ++ir_c_;\n";
         s += "            }\n        }\n        ir_cnt_[ir_p_] = ir_c_;\n    }\n";
         snprintf(buf, sizeof(buf),
@@ -517,7 +524,7 @@ std::string generate(const beast_ir *ir) {
         s += buf;
         for (int l = 0; l < nck; ++l) {
             snprintf(buf, sizeof(buf),
-                     "    { const u64 ir_x_ = warp_sum(ir_rej_[%d]); if (ir_lane_ == 0 && ir_x_) atomicAdd(&ir_stats_[NI + %d], ir_x_); }\n",
+                     "    { const u64 ir_x_ = warp_sum(ir_rej%d_); if (ir_lane_ == 0 && ir_x_) atomicAdd(&ir_stats_[NI + %d], ir_x_); }\n",
                      l, idx[l]);
             s += buf;
         }
@@ -539,6 +546,66 @@ std::string generate(const beast_ir *ir) {
             s += buf;
         }
         s += "                    ++ir_pos_;\n                }\n            }\n        }\n    }\n}\n";
+        // warp-per-parent fused pair: lanes take the level-k values, each
+        // lane runs the level-(k+1) loop of its value (uniform trip counts
+        // when the inner range does not depend on the outer value)
+        const std::string whead =
+            "    const unsigned ir_lane_ = threadIdx.x & 31;\n"
+            "    const u64 ir_w0_ = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;\n"
+            "    const u64 ir_nw_ = ((u64)gridDim.x * blockDim.x) >> 5;\n";
+        snprintf(buf, sizeof(buf),
+                 "extern \"C\" __global__ void __launch_bounds__(256) ir_wfcount_%d(const i64 *ir_par_, u64 ir_npar_, "
+                 "u64 *ir_cnt_, u64 *ir_stats_) {\n", k);
+        s += buf;
+        s += whead + consts;
+        s += "    u64 ir_vis_ = 0, ir_vis2_ = 0;\n" + rej_decl(nck);
+        s += "    for (u64 ir_p_ = ir_w0_; ir_p_ < ir_npar_; ir_p_ += ir_nw_) {\n" + parent;
+        s += "        ir_vis_ += ir_n_;\n        u64 ir_c_ = 0;\n";
+        s += "        for (u64 ir_i_ = ir_lane_; ir_i_ < ir_n_; ir_i_ += 32) {\n" + outer;
+        s += "            ir_vis2_ += ir_n2_;\n";
+        s += "            for (u64 ir_j_ = 0; ir_j_ < ir_n2_; ++ir_j_) {\n" + inner;
+        if (nck) s += rej_inc(nck, "                ");
+        else s += "                ++ir_c_;\n";
+        s += "            }\n        }\n        ir_c_ = warp_sum(ir_c_);\n        if (ir_lane_ == 0) ir_cnt_[ir_p_] = ir_c_;\n    }\n";
+        snprintf(buf, sizeof(buf),
+                 "    if (ir_lane_ == 0 && ir_vis_) atomicAdd(&ir_stats_[%d], ir_vis_);\n"
+                 "    ir_vis2_ = warp_sum(ir_vis2_);\n    if (ir_lane_ == 0 && ir_vis2_) atomicAdd(&ir_stats_[%d], ir_vis2_);\n",
+                 k, k + 1);
+        s += buf;
+        for (int l = 0; l < nck; ++l) {
+            snprintf(buf, sizeof(buf),
+                     "    { const u64 ir_x_ = warp_sum(ir_rej%d_); if (ir_lane_ == 0 && ir_x_) atomicAdd(&ir_stats_[NI + %d], ir_x_); }\n",
+                     l, idx[l]);
+            s += buf;
+        }
+        s += "}\n";
+        snprintf(buf, sizeof(buf),
+                 "extern \"C\" __global__ void __launch_bounds__(256) ir_wfemit_%d(const i64 *ir_par_, u64 ir_npar_, "
+                 "const u64 *ir_off_, i64 *ir_out_) {\n", k);
+        s += buf;
+        s += whead + consts;
+        s += "    for (u64 ir_p_ = ir_w0_; ir_p_ < ir_npar_; ir_p_ += ir_nw_) {\n" + parent;
+        s += "        u64 ir_pos_ = ir_off_[ir_p_];\n";
+        s += "        for (u64 ir_b_ = 0; ir_b_ < ir_n_; ir_b_ += 32) {\n";
+        s += "            const u64 ir_i_ = ir_b_ + ir_lane_;\n            u64 ir_k_ = 0;\n";
+        s += "            if (ir_i_ < ir_n_) {\n" + outer;
+        s += "            for (u64 ir_j_ = 0; ir_j_ < ir_n2_; ++ir_j_) {\n" + inner;
+        s += "                if (ir_r_ == 0) ++ir_k_;\n            }\n            }\n";
+        // warp exclusive scan of the lanes' survivor counts (lane order = value order of level k)
+        s += "            u64 ir_x_ = ir_k_;\n";
+        s += "            for (int ir_o_ = 1; ir_o_ < 32; ir_o_ <<= 1) { const u64 ir_y_ = __shfl_up_sync(0xffffffffu, ir_x_, ir_o_); if ((int)ir_lane_ >= ir_o_) ir_x_ += ir_y_; }\n";
+        s += "            const u64 ir_tot_ = __shfl_sync(0xffffffffu, ir_x_, 31);\n";
+        s += "            if (ir_k_) {\n                u64 ir_q_ = ir_pos_ + ir_x_ - ir_k_;\n" + outer;
+        s += "            for (u64 ir_j_ = 0; ir_j_ < ir_n2_; ++ir_j_) {\n" + inner;
+        s += "                if (ir_r_ == 0) {\n";
+        snprintf(buf, sizeof(buf), "                    i64 *ir_row_ = ir_out_ + ir_q_ * %du;\n", k + 2);
+        s += buf;
+        for (int j = 0; j <= k + 1; ++j) {
+            snprintf(buf, sizeof(buf), "                    ir_row_[%d] = %s;\n", j, ir->inames[j].c_str());
+            s += buf;
+        }
+        s += "                    ++ir_q_;\n                }\n            }\n            }\n";
+        s += "            ir_pos_ += ir_tot_;\n        }\n    }\n}\n";
     }
     return s;
 }
@@ -600,6 +667,8 @@ int load(beast_ir *ir) {
     }
     ir->k_fcount.assign(ir->ni, nullptr);
     ir->k_femit.assign(ir->ni, nullptr);
+    ir->k_wfcount.assign(ir->ni, nullptr);
+    ir->k_wfemit.assign(ir->ni, nullptr);
     for (int k = 0; k + 1 < ir->ni; ++k) {
         // fuse (k, k + 1) where level k has no constraints and level k + 1
         // filters (or is the deepest): its rows are the ones materialised
@@ -611,6 +680,8 @@ int load(beast_ir *ir) {
         if (!free_k || !filters) continue;
         IRCK(cudaLibraryGetKernel(&ir->k_fcount[k], ir->lib, ("ir_fcount_" + std::to_string(k)).c_str()));
         IRCK(cudaLibraryGetKernel(&ir->k_femit[k], ir->lib, ("ir_femit_" + std::to_string(k)).c_str()));
+        IRCK(cudaLibraryGetKernel(&ir->k_wfcount[k], ir->lib, ("ir_wfcount_" + std::to_string(k)).c_str()));
+        IRCK(cudaLibraryGetKernel(&ir->k_wfemit[k], ir->lib, ("ir_wfemit_" + std::to_string(k)).c_str()));
     }
     IRCK(cudaLibraryGetKernel(&ir->k_tiles, ir->lib, "ir_scan_tiles"));
     IRCK(cudaLibraryGetKernel(&ir->k_top, ir->lib, "ir_scan_top"));
@@ -686,9 +757,41 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
     // this many parents (BEAST_IR_FUSE_MIN, default 8 x 8 CTAs x 256 threads per SM)
     unsigned long long fuse_min = 8ull * grid * 256;
     if (const char *e = getenv("BEAST_IR_FUSE_MIN")) fuse_min = strtoull(e, nullptr, 10);
+    // BEAST_IR_TRACE=1: per-level step time and shape on stderr (development)
+    const bool trace = getenv("BEAST_IR_TRACE") != nullptr;
+    cudaEvent_t tev[2] = {nullptr, nullptr};
+    if (trace) {
+        cudaEventCreate(&tev[0]);
+        cudaEventCreate(&tev[1]);
+    }
     for (int k = 0; k < NI && n_par;) {
-        const bool fused = ir->k_fcount[k] != nullptr && n_par >= fuse_min;
+        if (trace) cudaEventRecord(tev[0], st);
+        const unsigned long long n_par_in = n_par;
+        bool fused = ir->k_fcount[k] != nullptr && n_par >= fuse_min;
         const bool tmode = n_par >= thread_min;
+        if (!fused && ir->k_fcount[k] != nullptr) {
+            // would level k's rows be large?  count them (level k has no
+            // constraints: the children are its trip counts) and fuse with
+            // k + 1 instead of materialising more than BEAST_IR_MATERIALIZE_MAX
+            // bytes (default 256 MiB)
+            unsigned long long lim = 256ull << 20;
+            if (const char *e = getenv("BEAST_IR_MATERIALIZE_MAX")) lim = strtoull(e, nullptr, 10);
+            unsigned long long *cnt0 = nullptr, *stats0 = nullptr;
+            IRCK(cudaMallocAsync((void **)&cnt0, (n_par + 1) * 8, st));
+            IRCK(cudaMallocAsync((void **)&stats0, (size_t)(NI + NC + 1) * 8, st));   // scratch statistics
+            const long long *pc = par;
+            void *a[] = {(void *)&pc, (void *)&n_par, (void *)&cnt0, (void *)&stats0};
+            rc = launch(ir, tmode ? ir->k_tcount[k] : ir->k_count[k], grid, 256, st, a);
+            unsigned long long *off0 = nullptr, kids = 0;
+            if (rc == BEAST_OK) IRCK(cudaMallocAsync((void **)&off0, (n_par + 1) * 8, st));
+            if (rc == BEAST_OK) rc = scan(ir, cnt0, n_par, off0, st, &kids);
+            cudaFreeAsync(cnt0, st);
+            cudaFreeAsync(stats0, st);
+            if (off0) cudaFreeAsync(off0, st);
+            if (rc != BEAST_OK) break;
+            fused = kids * (unsigned long long)(k + 1) * 8 > lim;
+        }
+        const bool wfused = fused && !tmode;   // warp per parent unless there are very many parents
         const int k_last = fused ? k + 1 : k;   // deepest level of this step
         unsigned long long *cnt = nullptr, *off = nullptr;
         IRCK(cudaMallocAsync((void **)&cnt, (n_par + 1) * 8, st));
@@ -696,7 +799,8 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
         {
             const long long *pc = par;
             void *a[] = {(void *)&pc, (void *)&n_par, (void *)&cnt, (void *)&stats};
-            rc = launch(ir, fused ? ir->k_fcount[k] : tmode ? ir->k_tcount[k] : ir->k_count[k], grid, 256, st, a);
+            rc = launch(ir, wfused ? ir->k_wfcount[k] : fused ? ir->k_fcount[k] : tmode ? ir->k_tcount[k] : ir->k_count[k],
+                        grid, 256, st, a);
         }
         if (rc == BEAST_OK) rc = scan(ir, cnt, n_par, off, st, &total);
         long long *child = nullptr;
@@ -716,7 +820,8 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
             if (rc == BEAST_OK) {
                 const long long *pc = par;
                 void *a[] = {(void *)&pc, (void *)&n_par, (void *)&off, (void *)&child};
-                rc = launch(ir, fused ? ir->k_femit[k] : tmode ? ir->k_temit[k] : ir->k_emit[k], grid, 256, st, a);
+                rc = launch(ir, wfused ? ir->k_wfemit[k] : fused ? ir->k_femit[k] : tmode ? ir->k_temit[k] : ir->k_emit[k],
+                            grid, 256, st, a);
             }
         }
         cudaFreeAsync(cnt, st);
@@ -724,11 +829,23 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
         if (par) cudaFreeAsync(par, st);
         par = (last || rc != BEAST_OK) ? nullptr : child;
         n_par = total;
+        if (trace) {
+            float ms = 0;
+            cudaEventRecord(tev[1], st);
+            cudaEventSynchronize(tev[1]);
+            cudaEventElapsedTime(&ms, tev[0], tev[1]);
+            fprintf(stderr, "ir level %d%s%s: parents %llu -> children %llu  %.4f ms\n", k, fused ? "+1 (fused)" : "",
+                    tmode ? " thread/parent" : " warp/parent", n_par_in, total, ms);
+        }
         if (rc != BEAST_OK) {
             if (child && child != out) cudaFreeAsync(child, st);
             break;
         }
         k = k_last + 1;
+    }
+    if (trace) {
+        cudaEventDestroy(tev[0]);
+        cudaEventDestroy(tev[1]);
     }
     if (NI == 0) total = pruned ? 0 : 1;
     std::vector<unsigned long long> h(NI + NC);

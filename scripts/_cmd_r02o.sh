@@ -1,0 +1,7 @@
+for v in "" variants/pc1500.so; do
+  echo "== ${v:-default}"
+  BEAST_LIB_PATH=$v python scripts/shard_time.py b200_S 8 2>&1 | tail -3
+  BEAST_LIB_PATH=$v python scripts/shard_time.py b200_C 8 2>&1 | tail -1
+  BEAST_LIB_PATH=$v python scripts/shard_time.py b200_D 8 2>&1 | tail -1
+  BEAST_LIB_PATH=$v python scripts/shard_time.py headline 20 2>&1 | tail -1
+done

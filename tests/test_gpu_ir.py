@@ -106,12 +106,16 @@ class _Env:
     """Force the engine's alternative kernel shapes (read by each run): the
     thread-per-parent kernels on every level (BEAST_IR_THREAD_MIN = 0) and/or
     the fused two-level kernels wherever a level has no constraints
-    (BEAST_IR_FUSE_MIN = 0) -- by default they serve only levels with many
-    parents, which the small parity spaces never reach."""
+    (BEAST_IR_FUSE_MIN = 0: warp per parent; with BEAST_IR_THREAD_MIN = 0:
+    thread per parent), or the fusion the engine chooses when a level's rows
+    would exceed BEAST_IR_MATERIALIZE_MAX bytes (0: always) -- by default
+    they serve only levels with many parents or rows, which the small parity
+    spaces never reach."""
 
     MODES = {"thread": {"BEAST_IR_THREAD_MIN": "0"},
-             "fused": {"BEAST_IR_FUSE_MIN": "0"},
-             "fused_thread": {"BEAST_IR_THREAD_MIN": "0", "BEAST_IR_FUSE_MIN": "0"}}
+             "fused": {"BEAST_IR_FUSE_MIN": "0"},                  # warp per parent, fused pairs
+             "fused_thread": {"BEAST_IR_THREAD_MIN": "0", "BEAST_IR_FUSE_MIN": "0"},
+             "adaptive": {"BEAST_IR_MATERIALIZE_MAX": "0"}}        # fuse wherever rows would materialise
 
     def __init__(self, mode):
         self.vars = self.MODES[mode]
