@@ -1,0 +1,2 @@
+timeout 900 python -m pytest -x -q tests/test_gpu_parity.py -k "tiny or micro or headline or full_size or fuzz or virtual" 2>&1 | tail -2
+bash scripts/ab2.sh "headline b200_S" variants/tm32.so variants/tm256.so variants/tmoff.so
