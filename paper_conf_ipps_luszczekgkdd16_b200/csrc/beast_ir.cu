@@ -401,7 +401,7 @@ std::string generate(const beast_ir *ir) {
         s += buf;
         s += head + consts;
         s += "    for (u64 ir_p_ = ir_w0_; ir_p_ < ir_npar_; ir_p_ += ir_nw_) {\n" + parent;
-        s += "        u64 ir_pos_ = ir_off_[ir_p_];\n";
+        s += "        u64 ir_pos_ = ir_off_[ir_p_];\n        if (ir_off_[ir_p_ + 1] == ir_pos_) continue;   // no children: nothing to re-evaluate\n";
         s += "        for (u64 ir_b_ = 0; ir_b_ < ir_n_; ir_b_ += 32) {\n";
         s += "            const u64 ir_i_ = ir_b_ + ir_lane_;\n            bool ir_keep_ = false;\n";
         s += "            if (ir_i_ < ir_n_) {\n" + point + "            ir_keep_ = ir_r_ == 0;\n            }\n";
@@ -453,7 +453,7 @@ std::string generate(const beast_ir *ir) {
         s += buf;
         s += thead + consts + "    (void)ir_lane_;\n";
         s += "    for (u64 ir_p_ = ir_t0_; ir_p_ < ir_npar_; ir_p_ += ir_nt_) {\n" + parent;
-        s += "        u64 ir_pos_ = ir_off_[ir_p_];\n";
+        s += "        u64 ir_pos_ = ir_off_[ir_p_];\n        if (ir_off_[ir_p_ + 1] == ir_pos_) continue;   // no children: nothing to re-evaluate\n";
         s += "        for (u64 ir_i_ = 0; ir_i_ < ir_n_; ++ir_i_) {\n" + point;
         s += "            if (ir_r_ == 0) {\n";
         snprintf(buf, sizeof(buf), "                i64 *ir_row_ = ir_out_ + ir_pos_ * %du;\n", k + 1);
@@ -547,7 +547,7 @@ std::string generate(const beast_ir *ir) {
         s += buf;
         s += thead + consts + "    (void)ir_lane_;\n";
         s += "    for (u64 ir_p_ = ir_t0_; ir_p_ < ir_npar_; ir_p_ += ir_nt_) {\n" + parent;
-        s += "        u64 ir_pos_ = ir_off_[ir_p_];\n";
+        s += "        u64 ir_pos_ = ir_off_[ir_p_];\n        if (ir_off_[ir_p_ + 1] == ir_pos_) continue;   // no children: nothing to re-evaluate\n";
         s += "        for (u64 ir_i_ = 0; ir_i_ < ir_n_; ++ir_i_) {\n" + outer;
         s += "            for (u64 ir_j_ = 0; ir_j_ < ir_n2_; ++ir_j_) {\n" + inner;
         s += "                if (ir_r_ == 0) {\n";
@@ -614,7 +614,7 @@ std::string generate(const beast_ir *ir) {
         s += buf;
         s += whead + consts;
         s += "    for (u64 ir_p_ = ir_w0_; ir_p_ < ir_npar_; ir_p_ += ir_nw_) {\n" + parent + choose;
-        s += "        u64 ir_pos_ = ir_off_[ir_p_];\n";
+        s += "        u64 ir_pos_ = ir_off_[ir_p_];\n        if (ir_off_[ir_p_ + 1] == ir_pos_) continue;   // no children: nothing to re-evaluate\n";
         // lanes over level k+1: ballot-ranked rows, value by value
         s += "        if (ir_inner_) {\n";
         s += "        for (u64 ir_i_ = 0; ir_i_ < ir_n_; ++ir_i_) {\n" + outer;
