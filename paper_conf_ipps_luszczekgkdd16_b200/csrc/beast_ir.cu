@@ -190,7 +190,6 @@ struct beast_ir {
     std::vector<cudaKernel_t> k_tcount, k_temit;   // per level, thread per parent
     std::vector<cudaKernel_t> k_fcount, k_femit;   // levels k and k + 1 fused (k without constraints), else null
     std::vector<cudaKernel_t> k_wfcount, k_wfemit; // the same, warp per parent
-    std::vector<cudaKernel_t> k_probe;             // per level, mean trip count over a sample of parents
     cudaKernel_t k_root = nullptr, k_tiles = nullptr, k_top = nullptr,
                  k_add = nullptr;
     int sm_count = 148;
@@ -466,17 +465,7 @@ std::string generate(const beast_ir *ir) {
                  ir->inames[k].c_str());
         s += buf;
         s += "            }\n        }\n    }\n}\n";
-        // trip-count probe: the mean range length of level k over a sample of
-        // parents (the engine picks warp or thread per parent from it)
-        snprintf(buf, sizeof(buf),
-                 "extern \"C\" __global__ void __launch_bounds__(256) ir_probe_%d(const i64 *ir_par_, u64 ir_npar_, "
-                 "u64 ir_stride_, u64 ir_ns_, u64 *ir_sum_) {\n", k);
-        s += buf;
-        s += consts;
-        s += "    const u64 ir_s_ = (u64)blockIdx.x * blockDim.x + threadIdx.x;\n    u64 ir_t_ = 0;\n";
-        s += "    if (ir_s_ < ir_ns_) {\n        const u64 ir_p_ = ir_s_ * ir_stride_;\n" + parent;
-        s += "        ir_t_ = ir_n_;\n    }\n    ir_t_ = warp_sum(ir_t_);\n";
-        s += "    if ((threadIdx.x & 31) == 0 && ir_t_) atomicAdd(ir_sum_, ir_t_);\n}\n";
+
     }
     // Fused pairs (k, k + 1) for a level k without constraints: one thread per
     // parent runs both loops (the level-(k+1) range re-evaluated per value of
@@ -707,13 +696,11 @@ int load(beast_ir *ir) {
     ir->k_emit.assign(ir->ni, nullptr);
     ir->k_tcount.assign(ir->ni, nullptr);
     ir->k_temit.assign(ir->ni, nullptr);
-    ir->k_probe.assign(ir->ni, nullptr);
     for (int k = 0; k < ir->ni; ++k) {
         IRCK(cudaLibraryGetKernel(&ir->k_count[k], ir->lib, ("ir_count_" + std::to_string(k)).c_str()));
         IRCK(cudaLibraryGetKernel(&ir->k_emit[k], ir->lib, ("ir_emit_" + std::to_string(k)).c_str()));
         IRCK(cudaLibraryGetKernel(&ir->k_tcount[k], ir->lib, ("ir_tcount_" + std::to_string(k)).c_str()));
         IRCK(cudaLibraryGetKernel(&ir->k_temit[k], ir->lib, ("ir_temit_" + std::to_string(k)).c_str()));
-        IRCK(cudaLibraryGetKernel(&ir->k_probe[k], ir->lib, ("ir_probe_" + std::to_string(k)).c_str()));
     }
     ir->k_fcount.assign(ir->ni, nullptr);
     ir->k_femit.assign(ir->ni, nullptr);
@@ -802,15 +789,8 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
     // thread per parent once the parents outnumber the resident threads many
     // times over (BEAST_IR_THREAD_MIN, default 64 x 8 CTAs x 256 threads per SM)
     unsigned long long thread_min = 64ull * grid * 256;
-    const char *thread_min_env = getenv("BEAST_IR_THREAD_MIN");
-    if (thread_min_env) thread_min = strtoull(thread_min_env, nullptr, 10);
-    // otherwise a level with many parents (>= BEAST_IR_PROBE_MIN, 65536)
-    // samples 4096 of them: a mean range shorter than 16 values takes one
-    // thread per parent (a warp per parent would leave most lanes idle)
-    unsigned long long probe_min = 65536;
-    if (const char *e = getenv("BEAST_IR_PROBE_MIN")) probe_min = strtoull(e, nullptr, 10);
-    unsigned long long *probe_sum = nullptr;
-    IRCK(cudaMallocAsync((void **)&probe_sum, 8, st));
+    if (const char *e = getenv("BEAST_IR_THREAD_MIN")) thread_min = strtoull(e, nullptr, 10);
+
     // levels k, k + 1 fused (level k has no constraints) once level k has
     // this many parents (BEAST_IR_FUSE_MIN, default 8 x 8 CTAs x 256 threads per SM)
     unsigned long long fuse_min = 8ull * grid * 256;
@@ -826,19 +806,8 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
         if (trace) cudaEventRecord(tev[0], st);
         const unsigned long long n_par_in = n_par;
         bool fused = ir->k_fcount[k] != nullptr && n_par >= fuse_min;
-        bool tmode = n_par >= thread_min;
-        if (!thread_min_env && !tmode && n_par >= probe_min) {
-            const unsigned long long ns = 4096, stride = n_par / ns;
-            IRCK(cudaMemsetAsync(probe_sum, 0, 8, st));
-            const long long *pc = par;
-            void *a[] = {(void *)&pc, (void *)&n_par, (void *)&stride, (void *)&ns, (void *)&probe_sum};
-            rc = launch(ir, ir->k_probe[k], (unsigned)(ns / 256), 256, st, a);
-            if (rc != BEAST_OK) break;
-            unsigned long long sum = 0;
-            IRCK(cudaMemcpyAsync(&sum, probe_sum, 8, cudaMemcpyDeviceToHost, st));
-            IRCK(cudaStreamSynchronize(st));
-            tmode = sum < 16 * ns;
-        }
+        const bool tmode = n_par >= thread_min;
+
         if (!fused && ir->k_fcount[k] != nullptr) {
             // would level k's rows be large?  count them (level k has no
             // constraints: the children are its trip counts) and fuse with
@@ -917,7 +886,6 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
         cudaEventDestroy(tev[0]);
         cudaEventDestroy(tev[1]);
     }
-    cudaFreeAsync(probe_sum, st);
     if (NI == 0) total = pruned ? 0 : 1;
     std::vector<unsigned long long> h(NI + NC);
     if (NI + NC) IRCK(cudaMemcpyAsync(h.data(), stats, (size_t)(NI + NC) * 8, cudaMemcpyDeviceToHost, st));

@@ -1,0 +1,4 @@
+timeout 900 python -m pytest -x -q tests/test_gpu_parity.py -k "tiny or micro or headline or full_size or fuzz or virtual or async or host" tests/test_gpu_fused_gather.py tests/test_gpu_ir.py 2>&1 | tail -2
+bash scripts/ab2.sh "headline b200_S" variants/noF.so
+bash scripts/ab2.sh "headline b200_S" variants/noF.so
+BEAST_IR_TRACE=1 python scripts/ir_time.py headline 2>&1 | tail -16
