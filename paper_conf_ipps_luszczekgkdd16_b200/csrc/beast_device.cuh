@@ -241,10 +241,13 @@ __device__ __forceinline__ uint32_t scan_rows(uint32_t s1, uint32_t s2, uint32_t
 }
 
 // The same scan in the instrumented build: `blocks` is incremented inside
-// the loop body, once per executed 16-point iteration (beast_stats.formed).
-// (A separate function, so the timed kernels keep scan_rows' exact code.)
+// the loop body, once per executed 16-point iteration b < nb_own
+// (beast_stats.formed; nb_own = ceil(L / 16) of the lane's own rows, which is
+// below the warp's NB when the warp's rows come from jobs of different
+// lengths).  (A separate function, so the timed kernels keep scan_rows'
+// exact code.)
 __device__ __forceinline__ uint32_t scan_rows_counted(uint32_t s1, uint32_t s2, uint32_t T, uint32_t NB,
-                                                      uint32_t &blocks) {
+                                                      uint32_t nb_own, uint32_t &blocks) {
     const uint32_t Sp = s1 | (s2 << 16);
     uint32_t Cb = (0x10000u - T) * 0x10001u;
     asm volatile("" : "+r"(Cb));
@@ -258,7 +261,8 @@ __device__ __forceinline__ uint32_t scan_rows_counted(uint32_t s1, uint32_t s2, 
     for (uint32_t b = 0; b < NB; ++b) {
         eval16pp<KI>(acc, acc2, Cb, Sp, M);
         Cb += step;
-        asm volatile("add.u32 %0, %0, 1;" : "+r"(blocks));   // counted where the block runs
+        asm volatile("{\n\t.reg .pred p;\n\tsetp.lt.u32 p, %1, %2;\n\t@p add.u32 %0, %0, 1;\n\t}"
+                     : "+r"(blocks) : "r"(b), "r"(nb_own));   // counted where the block runs
     }
     return vmin_u16x2(acc, acc2);
 }
