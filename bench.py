@@ -518,7 +518,10 @@ def main():
             "count": count_line,
             "replicas": {"l4_digests": ["0x%016x" % d for d in replicas], "ranks_agree": len(set(replicas)) == 1,
                          "how": "digest of each rank's redundantly computed L1-L4 list, all-gathered"},
-            "roofline": {"bound": "alu", "kernel": "k_eval<A> (L8-L9 A-read grids)",
+            "roofline": {"bound": "alu",
+                         "kernel": "k_tile_eval<A> (L8-L9 A-read grids; each 512-prefix tile is bucketed by row "
+                                   "length in shared memory by the same kernel, so its time includes the "
+                                   "flattening that round 1 ran as two separate kernels)",
                          "achieved": achieved / 1e12, "peak": peak_ops / 1e12, "unit": "T int16-ops/s",
                          "frac": achieved / peak_ops if peak_ops else None, "traffic": traffic,
                          "peak_measured_scan": scan_ceiling_ops / 1e12,
@@ -530,7 +533,11 @@ def main():
                          "avg_launch_ms": a_ms,
                          "peak_source": "%d SMs x %d int lane-instr/clk x 2 (16-bit halves) x sm_max_mhz (%s "
                                         "MEASURED_PEAKS.json); 2 int ops per point" % (sm_count, lanes, peak_src),
-                         "points_per_s_kernel": a_points / (a_ms / 1e3) if a_ms > 0 else None},
+                         "points_per_s_kernel": a_points / (a_ms / 1e3) if a_ms > 0 else None,
+                         "frac_whole_pass": (n_canon / (ms / 1e3)) / (peak_ops / ops_per_point)
+                         if peak_ops else None,
+                         "frac_whole_pass_how": "canonical points per second of the whole step (all 15 levels, "
+                                                "every kernel) against the same peak, one point = 2 ops"},
             "e2e": {"value": n_canon / (e2e_step / 1e3), "unit": UNIT,
                     "h2d_bytes_per_step": 0,
                     "inputs": "a 96-byte space description, resolved into kernel parameters when the handle "
@@ -551,7 +558,7 @@ def main():
             "cpu_baseline": cpu,
             "stages_ms": stages,
             "timing": "value: per-step CUDA events around beast_enumerate_async passes (device time, L2 "
-                      "flushed before each step, counts checked after the loop); roofline: k_eval<A> "
+                      "flushed before each step, counts checked after the loop); roofline: k_tile_eval<A> "
                       "launches timed by CUDA events in a second loop of synchronous flushed steps",
             "factorised": fact,
             "sweep": sweep,

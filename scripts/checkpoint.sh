@@ -15,11 +15,11 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --profile-
   --log-file gpurun_out/${TAG}_headline_launches.csv python scripts/prof_run.py headline > /dev/null 2>&1
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --profile-from-start off --csv \
   --log-file gpurun_out/${TAG}_b200_S_launches.csv python scripts/prof_run.py b200_S > /dev/null 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on --profile-from-start off -k regex:k_eval -c 2 \
+timeout 900 ncu --set full --clock-control none --import-source on --profile-from-start off -k regex:"k_tile_eval|k_place_write|k_scan_lb" -c 4 \
   -o gpurun_out/${TAG}_headline_keval python scripts/prof_run.py headline > gpurun_out/${TAG}_ncu_keval.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on --profile-from-start off -k regex:k_seg_level -c 3 \
   -o gpurun_out/${TAG}_headline_seglvl python scripts/prof_run.py headline > gpurun_out/${TAG}_ncu_seglvl.log 2>&1
-timeout 900 ncu --set full --clock-control none --profile-from-start off -k regex:k_eval -c 1 \
+timeout 900 ncu --set full --clock-control none --profile-from-start off -k regex:k_tile_eval -c 2 \
   -o gpurun_out/${TAG}_b200_S_keval python scripts/prof_run.py b200_S > gpurun_out/${TAG}_ncu_keval_S.log 2>&1
 for r in headline_keval headline_seglvl b200_S_keval; do
   ncu -i gpurun_out/${TAG}_$r.ncu-rep --page raw --csv > gpurun_out/${TAG}_${r}_raw.csv 2>/dev/null

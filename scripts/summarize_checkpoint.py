@@ -1,6 +1,6 @@
 """Write profiles/<TAG>_*.md from a scripts/checkpoint.sh run's gpurun_out/
 files: the launch lists (headline, SGEMM-B200), the ncu --set full metrics of
-k_eval and the prefix-stage levels, and the bench lines' key numbers.
+k_tile_eval<A>/<B>, the tail kernels and the prefix-stage levels, and the bench lines' key numbers.
 Usage: python scripts/summarize_checkpoint.py TAG"""
 import csv
 import json
@@ -47,7 +47,8 @@ def main():
                                 capture_output=True, text=True).stdout
             parts.append("## Launch list, %s (ncu `gpu__time_duration.sum --clock-control none`, one pass of "
                          "`scripts/prof_run.py %s`; cold-cache and serialised: compare shares)\n\n%s" % (wl, wl, md))
-    for r, what in (("headline_keval", "k_eval<A>, k_eval<B>, headline"), ("b200_S_keval", "k_eval<A>, SGEMM-B200"),
+    for r, what in (("headline_keval", "k_tile_eval<A>, k_tile_eval<B>, scan, placement + write-out, headline"),
+                    ("b200_S_keval", "k_tile_eval<A>, k_tile_eval<B>, SGEMM-B200"),
                     ("headline_seglvl", "prefix-stage levels, headline")):
         p = os.path.join(OUT, "%s_%s_raw.csv" % (tag, r))
         if os.path.exists(p):
@@ -60,7 +61,7 @@ def main():
             except Exception:
                 continue
             r = d["roofline"]
-            parts.append("## bench line, %s\n\nms/step %.4f, value %.4g points/s, k_eval<A> %.4f ms = %.3f of the derived "
+            parts.append("## bench line, %s\n\nms/step %.4f, value %.4g points/s, k_tile_eval<A> %.4f ms = %.3f of the derived "
                          "issue peak, %.3f of the measured packed-scan ceiling; count %.4f ms; e2e %.4g points/s; "
                          "write-out %s; clocks %s\n" % (
                              wl, d["ms_per_step"], d["value"], r["avg_launch_ms"], r["frac"], r["frac_measured_scan"],
