@@ -192,6 +192,12 @@ struct beast_ir {
     std::vector<cudaKernel_t> k_wfcount, k_wfemit; // the same, warp per parent
     cudaKernel_t k_root = nullptr, k_tiles = nullptr, k_top = nullptr,
                  k_add = nullptr;
+    // kernel-shape choices learnt from the previous run of this handle:
+    // average trip count of each level's iterator (values evaluated per
+    // parent; < 0: unknown) and the fuse decision of each fusable level
+    // (-1 unknown, 0 / 1)
+    std::vector<double> avg_trip;
+    std::vector<int> fuse_known;
     int sm_count = 148;
 };
 
@@ -340,8 +346,26 @@ std::string generate(const beast_ir *ir) {
     // root: constant-level constraints
     {
         std::vector<int> idx;
-        s += "extern \"C\" __global__ void ir_root(u64 *ir_stats_, int *ir_pruned_) {\n";
+        s += "extern \"C\" __global__ void ir_root(u64 *ir_stats_, int *ir_pruned_, u64 *ir_trip_) {\n";
         s += consts + derived_at(-1, -1, "    ");
+        // trip count of every iterator whose range depends on constants only
+        // (the engine runs such short levels one thread per parent)
+        for (int k = 0; k < ir->ni; ++k) {
+            bool constant = true;
+            for (const std::string *e : {&ir->istart[k], &ir->istop[k], &ir->istep[k]})
+                for (const std::string &id : idents(*e)) {
+                    bool ok = std::find(ir->cnames.begin(), ir->cnames.end(), id) != ir->cnames.end();
+                    for (size_t d = 0; d < ir->dnames.size() && !ok; ++d)
+                        ok = ir->dnames[d] == id && ir->dlev[d] < 0;
+                    constant = constant && ok;
+                }
+            if (constant)
+                s += "    { const i64 ir_st_ = (i64)(" + ir->istep[k] + "); ir_trip_[" + std::to_string(k) +
+                     "] = ir_st_ == 0 ? 0ull : ir_trip((i64)(" + ir->istart[k] + "), (i64)(" + ir->istop[k] +
+                     "), ir_st_); }\n";
+            else
+                s += "    ir_trip_[" + std::to_string(k) + "] = ~0ull;\n";
+        }
         s += "    int ir_r_ = 0;\n" + constraints_at(-1, "    ", &idx);
         s += "    int ir_g_ = 0;\n";
         for (size_t l = 0; l < idx.size(); ++l)
@@ -771,15 +795,18 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
     const int NI = ir->ni, NC = ir->nc;
     unsigned long long *stats = nullptr;
     int *pruned_d = nullptr;
-    IRCK(cudaMallocAsync((void **)&stats, (size_t)(NI + NC + 1) * 8, st));
+    IRCK(cudaMallocAsync((void **)&stats, (size_t)(NI + NC + 1 + NI) * 8, st));
     IRCK(cudaMemsetAsync(stats, 0, (size_t)(NI + NC + 1) * 8, st));
     pruned_d = (int *)(stats + NI + NC);
+    unsigned long long *trip_d = stats + NI + NC + 1;   // static trip count per iterator (~0: depends on the parent)
     {
-        void *a[] = {(void *)&stats, (void *)&pruned_d};
+        void *a[] = {(void *)&stats, (void *)&pruned_d, (void *)&trip_d};
         if (launch(ir, ir->k_root, 1, 1, st, a) != BEAST_OK) return BEAST_ERR_CUDA;
     }
     int pruned = 0;
+    std::vector<unsigned long long> trip(NI + 1, ~0ull);
     IRCK(cudaMemcpyAsync(&pruned, pruned_d, sizeof(int), cudaMemcpyDeviceToHost, st));
+    if (NI) IRCK(cudaMemcpyAsync(trip.data(), trip_d, (size_t)NI * 8, cudaMemcpyDeviceToHost, st));
     IRCK(cudaStreamSynchronize(st));
     unsigned long long n_par = pruned ? 0 : 1;
     long long *par = nullptr;   // level -1: one empty tuple
@@ -802,13 +829,26 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
         cudaEventCreate(&tev[0]);
         cudaEventCreate(&tev[1]);
     }
+    if ((int)ir->avg_trip.size() != NI) ir->avg_trip.assign(NI, -1.0);
+    if ((int)ir->fuse_known.size() != NI) ir->fuse_known.assign(NI, -1);
+    std::vector<unsigned long long> step_par(NI, 0);   // parents of the levels that start a step
     for (int k = 0; k < NI && n_par;) {
         if (trace) cudaEventRecord(tev[0], st);
         const unsigned long long n_par_in = n_par;
+        step_par[k] = n_par;
         bool fused = ir->k_fcount[k] != nullptr && n_par >= fuse_min;
-        const bool tmode = n_par >= thread_min;
+        if (!fused && ir->k_fcount[k] != nullptr && ir->fuse_known[k] >= 0) fused = ir->fuse_known[k] == 1;
+        // thread per parent: very many parents, or a level whose (constant)
+        // trip count is so short that a warp per parent would idle most lanes
+        // (BEAST_IR_SHORT_TRIP, default 8), given enough parents to fill the GPU
+        unsigned long long short_trip = 8;
+        if (const char *e = getenv("BEAST_IR_SHORT_TRIP")) short_trip = strtoull(e, nullptr, 10);
+        // the trip count: constant, else the previous run's average
+        const double trip_est = trip[k] != ~0ull ? (double)trip[k] : ir->avg_trip[k];
+        const bool tmode = n_par >= thread_min ||
+                           (trip_est >= 0 && trip_est <= (double)short_trip && n_par >= (unsigned long long)grid * 256);
 
-        if (!fused && ir->k_fcount[k] != nullptr) {
+        if (!fused && ir->k_fcount[k] != nullptr && ir->fuse_known[k] < 0) {
             // would level k's rows be large?  count them (level k has no
             // constraints: the children are its trip counts) and fuse with
             // k + 1 instead of materialising more than BEAST_IR_MATERIALIZE_MAX
@@ -829,6 +869,7 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
             if (off0) cudaFreeAsync(off0, st);
             if (rc != BEAST_OK) break;
             fused = kids * (unsigned long long)(k + 1) * 8 > lim;
+            ir->fuse_known[k] = fused ? 1 : 0;
         }
         const bool wfused = fused && !tmode;   // warp per parent unless there are very many parents
         const int k_last = fused ? k + 1 : k;   // deepest level of this step
@@ -892,6 +933,9 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
     IRCK(cudaFreeAsync(stats, st));
     IRCK(cudaStreamSynchronize(st));
     if (rc != BEAST_OK && rc != BEAST_ERR_CAPACITY) return rc;
+    if (rc == BEAST_OK)   // learn each step's trip counts for the next run
+        for (int i = 0; i < NI; ++i)
+            if (step_par[i]) ir->avg_trip[i] = (double)h[i] / (double)step_par[i];
     if (visits) for (int i = 0; i < NI; ++i) visits[i] = h[i];
     if (rejected) for (int i = 0; i < NC; ++i) rejected[i] = h[NI + i];
     if (written) *written = pruned ? 0 : total;
