@@ -631,7 +631,7 @@ def sweep_measure(beast, beast_inputs, stream, flush, reps=3):
             sp.close()
 
 
-def ir_measure(beast, desc, stream, flush, canonical_ms, reps=3):
+def ir_measure(beast, desc, stream, flush, canonical_ms, reps=7):
     """the same workload written in the generic space IR
     (tests/ir_specs.gemm_spec: Figs 11-15 as iterators, derived variables and
     constraints), compiled by the library with NVRTC and counted by the
@@ -664,6 +664,7 @@ def ir_measure(beast, desc, stream, flush, canonical_ms, reps=3):
         ms = []
         for _ in range(reps):
             flush.zero_()
+            torch.cuda.synchronize()   # the engine is host-driven (a sync per level): start it on an idle GPU
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a.record(stream)
             ir.count(stream=stream)
@@ -672,7 +673,8 @@ def ir_measure(beast, desc, stream, flush, canonical_ms, reps=3):
             ms.append(a.elapsed_time(b))
     m = statistics.median(ms)
     pts = sum(st["visits"])
-    return {"ms": m, "points": pts, "points_per_s": pts / (m / 1e3), "survivors": st["survivors"],
+    return {"ms": m, "ms_min": min(ms), "reps": reps, "points": pts, "points_per_s": pts / (m / 1e3),
+            "survivors": st["survivors"],
             "compile_s": compile_s, "vs_specialised": m / canonical_ms,
             "note": "generic IR engine (NVRTC-compiled, level-wise) on the same space; counting pass"}
 

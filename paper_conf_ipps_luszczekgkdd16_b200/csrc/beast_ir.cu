@@ -845,8 +845,10 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
         if (const char *e = getenv("BEAST_IR_SHORT_TRIP")) short_trip = strtoull(e, nullptr, 10);
         // the trip count: constant, else the previous run's average
         const double trip_est = trip[k] != ~0ull ? (double)trip[k] : ir->avg_trip[k];
+        const bool short_level = ir->k_fcount[k] == nullptr || !fused;   // (a fused step runs two loops)
         const bool tmode = n_par >= thread_min ||
-                           (trip_est >= 0 && trip_est <= (double)short_trip && n_par >= (unsigned long long)grid * 256);
+                           (short_level && trip_est >= 0 && trip_est <= (double)short_trip &&
+                            n_par >= (unsigned long long)grid * 256);
 
         if (!fused && ir->k_fcount[k] != nullptr && ir->fuse_known[k] < 0) {
             // would level k's rows be large?  count them (level k has no

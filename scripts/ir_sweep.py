@@ -21,6 +21,7 @@ with beast.Space.from_desc(desc) as sp:
     ref = sp.count(stats=True)[1]
 spec = ir_specs.gemm_spec(res, desc["precision"])
 stream = torch.cuda.current_stream().cuda_stream
+flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")   # L2 flush between reps, as bench.py
 with beast.IRSpace(spec) as ir:
     for v in vals:
         if v == "-":
@@ -30,12 +31,17 @@ with beast.IRSpace(spec) as ir:
         st = ir.count()
         ok = st["visits"] == ref["visits"] and st["rejected"] == ref["rejected"]
         ms = []
-        for _ in range(5):
+        for _ in range(int(os.environ.get("IR_REPS", "5"))):
+            if os.environ.get("IR_FLUSH", "1") == "1":
+                flush.zero_()
+            if os.environ.get("IR_SYNC", "0") == "1":
+                torch.cuda.synchronize()
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a.record()
             ir.count()
             b.record()
             torch.cuda.synchronize()
             ms.append(a.elapsed_time(b))
-        print("%s %s=%s: IR count %.3f ms (min %.3f) stats equal %s" % (name, var, v, statistics.median(ms), min(ms), ok),
+        print("%s %s=%s: IR count %.3f ms (min %.3f, all %s) stats equal %s" % (
+              name, var, v, statistics.median(ms), min(ms), ["%.2f" % x for x in ms], ok),
               flush=True)
