@@ -1,0 +1,52 @@
+"""Development: per-tile timeline of the three prefix levels from a
+BEAST_TILE_TRACE build (scripts/build_variant.sh trace -DBEAST_TILE_TRACE).
+Usage: BEAST_LIB_PATH=variants/trace.so python scripts/tile_trace.py [space]"""
+import ctypes
+import os
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import torch  # noqa: E402
+
+import beast_inputs as bi  # noqa: E402
+import paper_conf_ipps_luszczekgkdd16_b200 as beast  # noqa: E402
+from paper_conf_ipps_luszczekgkdd16_b200 import _lib  # noqa: E402
+
+name = sys.argv[1] if len(sys.argv) > 1 else "headline"
+sp = beast.Space.from_desc(bi.named(name))
+n = sp.count()
+out = torch.empty((max(n, 1), 2), dtype=torch.uint64, device="cuda")
+for _ in range(3):
+    beast.beast_enumerate(sp.handle, out)
+torch.cuda.synchronize()
+buf = np.zeros(3 * 8192 * 5, dtype=np.uint64)
+lib = ctypes.CDLL(_lib.LIB_PATH)
+assert lib.beast_debug_tile_trace(buf.ctypes.data_as(ctypes.c_void_p)) == 0
+tr = buf.reshape(3, 8192, 5).astype(np.int64)
+t0 = tr[0][tr[0][:, 0] > 0][:, 0].min()
+for lv, nm in enumerate(["L1-L3", "L4", "L5-L7"]):
+    t = tr[lv]
+    m = t[:, 0] > 0
+    t = t[m]
+    if not len(t):
+        continue
+    s, c, l, e = (t[:, i] - t0 for i in range(4))
+    print("%s: %d tiles, start %.1f..%.1f us, counted +%.2f us (med), looked back +%.2f us (med, max %.2f), "
+          "emitted +%.2f us (med, max %.2f), end of level %.1f us" % (
+              nm, len(t), s.min() / 1e3, s.max() / 1e3, np.median(c - s) / 1e3, np.median(l - c) / 1e3,
+              (l - c).max() / 1e3, np.median(e - l) / 1e3, (e - l).max() / 1e3, e.max() / 1e3))
+    order = np.argsort(s)
+    q = np.linspace(0, len(t) - 1, 9).astype(int)
+    print("   tile-ordered end times (us):", ["%.1f" % (e[i] / 1e3) for i in q])
+    print("   look-back done (us) at tile quantiles:", ["%.1f" % (l[i] / 1e3) for i in q])
+    print("   distinct CTAs %d, words max %d" % (len(set(t[:, 4] & 0xffffffff)), (t[:, 4] >> 32).max()))
+for lv in range(3):
+    t = tr[lv]
+    for k in range(3):
+        if t[k, 0] > 0:
+            print("level %d tile %d: start %.2f counted %.2f looked back %.2f emitted %.2f us, words %d" % (
+                lv, k, (t[k, 0] - t0) / 1e3, (t[k, 1] - t0) / 1e3, (t[k, 2] - t0) / 1e3, (t[k, 3] - t0) / 1e3,
+                t[k, 4] >> 32))
