@@ -50,3 +50,25 @@ for lv in range(3):
             print("level %d tile %d: start %.2f counted %.2f looked back %.2f emitted %.2f us, words %d" % (
                 lv, k, (t[k, 0] - t0) / 1e3, (t[k, 1] - t0) / 1e3, (t[k, 2] - t0) / 1e3, (t[k, 3] - t0) / 1e3,
                 t[k, 4] >> 32))
+
+# k_tile_eval timeline (last pass): reset the tile counter, run one pass, read
+tl = np.zeros(2 * 8192 * 3, dtype=np.uint64)
+ct = np.zeros(2 * 1024 * 2, dtype=np.uint64)
+lib.beast_debug_eval_trace(tl.ctypes.data_as(ctypes.c_void_p), ct.ctypes.data_as(ctypes.c_void_p))
+beast.beast_enumerate(sp.handle, out)
+torch.cuda.synchronize()
+lib.beast_debug_eval_trace(tl.ctypes.data_as(ctypes.c_void_p), ct.ctypes.data_as(ctypes.c_void_p))
+tl = tl.reshape(2, 8192, 3).astype(np.int64)
+ct = ct.reshape(2, 1024, 2).astype(np.int64)
+for st, nm in ((0, "A"), (1, "B")):
+    t = tl[st][tl[st][:, 0] > 0]
+    c = ct[st][ct[st][:, 0] > 0]
+    if not len(t):
+        continue
+    base = c[:, 0].min()
+    dur = (t[:, 1] - t[:, 0]) / 1e3
+    print("k_tile_eval<%s>: CTAs start %.1f..%.1f us, end %.1f..%.1f us; %d tiles, tile time med %.2f max %.2f us, "
+          "jobs med %d; first tile start %.1f, last tile end %.1f us" % (
+              nm, 0, (c[:, 0].max() - base) / 1e3, (c[:, 1].min() - base) / 1e3, (c[:, 1].max() - base) / 1e3,
+              len(t), np.median(dur), dur.max(), np.median(t[:, 2] >> 32), (t[:, 0].min() - base) / 1e3,
+              (t[:, 1].max() - base) / 1e3))
