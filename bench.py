@@ -471,7 +471,7 @@ def main():
         peaks, peak_src = _load_peaks()
         a_ms = statistics.mean(a_eval_ms)
         # survivor write-out (SURVEY §8(d) iii): 16 B per record written by
-        # k_write, against the HBM copy bandwidth of MEASURED_PEAKS.json
+        # k_place_write, against the HBM copy bandwidth of MEASURED_PEAKS.json
         w_ms = statistics.mean(write_ms) if write_ms and min(write_ms) > 0 else None
         w_bytes = 16 * st_local["survivors"]
         write_out = None
