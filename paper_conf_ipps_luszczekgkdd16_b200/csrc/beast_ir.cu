@@ -198,6 +198,12 @@ struct beast_ir {
     // (-1 unknown, 0 / 1)
     std::vector<double> avg_trip;
     std::vector<int> fuse_known;
+    // the previous run's level totals (children surviving through level k,
+    // ~0: not seen), its root pruning and static trip counts: a space is
+    // fixed, so a later run enqueues every level without waiting for the
+    // host (one synchronisation at the end, which checks these totals)
+    std::vector<unsigned long long> known_tot, known_trip;
+    int known_pruned = -1;
     int sm_count = 148;
 };
 
@@ -756,8 +762,10 @@ int launch(beast_ir *ir, cudaKernel_t k, unsigned grid, unsigned block, cudaStre
 }
 
 // Exclusive scan of n u64 counts into off[0..n] (off[n] = total); returns the total (host).
+// total == nullptr: no host copy and no synchronisation (the device total
+// is written to tot_dev).
 int scan(beast_ir *ir, const unsigned long long *cnt, unsigned long long n, unsigned long long *off,
-         cudaStream_t st, unsigned long long *total) {
+         cudaStream_t st, unsigned long long *total, unsigned long long *tot_dev) {
     const unsigned long long tiles = std::max(1ull, (n + 2047) / 2048);
     unsigned long long *ts = nullptr, *tot = nullptr;
     IRCK(cudaMallocAsync((void **)&ts, (tiles + 1) * 8, st));
@@ -776,14 +784,15 @@ int scan(beast_ir *ir, const unsigned long long *cnt, unsigned long long n, unsi
         void *a[] = {(void *)&off, (void *)&n, (void *)&ts, (void *)&tot};
         if (launch(ir, ir->k_add, g, 256, st, a) != BEAST_OK) return BEAST_ERR_CUDA;
     }
-    IRCK(cudaMemcpyAsync(total, tot, 8, cudaMemcpyDeviceToHost, st));
+    if (tot_dev) IRCK(cudaMemcpyAsync(tot_dev, tot, 8, cudaMemcpyDeviceToDevice, st));
+    if (total) IRCK(cudaMemcpyAsync(total, tot, 8, cudaMemcpyDeviceToHost, st));
     IRCK(cudaFreeAsync(ts, st));
-    IRCK(cudaStreamSynchronize(st));
+    if (total) IRCK(cudaStreamSynchronize(st));
     return BEAST_OK;
 }
 
 int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capacity, unsigned long long *written,
-        unsigned long long *visits, unsigned long long *rejected, bool emit_last) {
+        unsigned long long *visits, unsigned long long *rejected, bool emit_last, bool allow_replay = true) {
     const int lrc = load(ir);
     if (lrc != BEAST_OK) return lrc;
     int dev = 0;
@@ -795,19 +804,31 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
     const int NI = ir->ni, NC = ir->nc;
     unsigned long long *stats = nullptr;
     int *pruned_d = nullptr;
-    IRCK(cudaMallocAsync((void **)&stats, (size_t)(NI + NC + 1 + NI) * 8, st));
+    IRCK(cudaMallocAsync((void **)&stats, (size_t)(NI + NC + 1 + 2 * NI + 1) * 8, st));
     IRCK(cudaMemsetAsync(stats, 0, (size_t)(NI + NC + 1) * 8, st));
     pruned_d = (int *)(stats + NI + NC);
     unsigned long long *trip_d = stats + NI + NC + 1;   // static trip count per iterator (~0: depends on the parent)
+    unsigned long long *tot_d = trip_d + NI;             // device total of each step's deepest level
+    if (NI) IRCK(cudaMemsetAsync(tot_d, 0xff, (size_t)NI * 8, st));
     {
         void *a[] = {(void *)&stats, (void *)&pruned_d, (void *)&trip_d};
         if (launch(ir, ir->k_root, 1, 1, st, a) != BEAST_OK) return BEAST_ERR_CUDA;
     }
+    // replay: the previous run's totals stand in for the per-level host
+    // round trips (BEAST_IR_TRACE and the first run synchronise per level)
+    const bool trace_env = getenv("BEAST_IR_TRACE") != nullptr;
+    const bool replay = !trace_env && allow_replay && ir->known_pruned >= 0 && (int)ir->known_tot.size() == NI;
     int pruned = 0;
     std::vector<unsigned long long> trip(NI + 1, ~0ull);
-    IRCK(cudaMemcpyAsync(&pruned, pruned_d, sizeof(int), cudaMemcpyDeviceToHost, st));
-    if (NI) IRCK(cudaMemcpyAsync(trip.data(), trip_d, (size_t)NI * 8, cudaMemcpyDeviceToHost, st));
-    IRCK(cudaStreamSynchronize(st));
+    if (replay) {
+        pruned = ir->known_pruned;
+        for (int k = 0; k < NI; ++k) trip[k] = ir->known_trip[k];
+    } else {
+        IRCK(cudaMemcpyAsync(&pruned, pruned_d, sizeof(int), cudaMemcpyDeviceToHost, st));
+        if (NI) IRCK(cudaMemcpyAsync(trip.data(), trip_d, (size_t)NI * 8, cudaMemcpyDeviceToHost, st));
+        IRCK(cudaStreamSynchronize(st));
+    }
+    std::vector<unsigned long long> step_tot(NI, ~0ull);   // host totals of this run's steps (recording runs)
     unsigned long long n_par = pruned ? 0 : 1;
     long long *par = nullptr;   // level -1: one empty tuple
     int rc = BEAST_OK;
@@ -865,7 +886,7 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
             rc = launch(ir, tmode ? ir->k_tcount[k] : ir->k_count[k], grid, 256, st, a);
             unsigned long long *off0 = nullptr, kids = 0;
             if (rc == BEAST_OK) IRCK(cudaMallocAsync((void **)&off0, (n_par + 1) * 8, st));
-            if (rc == BEAST_OK) rc = scan(ir, cnt0, n_par, off0, st, &kids);
+            if (rc == BEAST_OK) rc = scan(ir, cnt0, n_par, off0, st, &kids, nullptr);
             cudaFreeAsync(cnt0, st);
             cudaFreeAsync(stats0, st);
             if (off0) cudaFreeAsync(off0, st);
@@ -884,7 +905,10 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
             rc = launch(ir, wfused ? ir->k_wfcount[k] : fused ? ir->k_fcount[k] : tmode ? ir->k_tcount[k] : ir->k_count[k],
                         grid, 256, st, a);
         }
-        if (rc == BEAST_OK) rc = scan(ir, cnt, n_par, off, st, &total);
+        const bool replay_step = replay && ir->known_tot[k_last] != ~0ull;
+        if (rc == BEAST_OK) rc = scan(ir, cnt, n_par, off, st, replay_step ? nullptr : &total, tot_d + k_last);
+        if (replay_step) total = ir->known_tot[k_last];
+        else step_tot[k_last] = total;
         long long *child = nullptr;
         const bool last = k_last == NI - 1;
         if (rc == BEAST_OK && (!last || emit_last) && total) {
@@ -930,10 +954,29 @@ int run(beast_ir *ir, cudaStream_t st, long long *out, unsigned long long capaci
         cudaEventDestroy(tev[1]);
     }
     if (NI == 0) total = pruned ? 0 : 1;
-    std::vector<unsigned long long> h(NI + NC);
+    std::vector<unsigned long long> h(NI + NC), dtot(NI, ~0ull);
     if (NI + NC) IRCK(cudaMemcpyAsync(h.data(), stats, (size_t)(NI + NC) * 8, cudaMemcpyDeviceToHost, st));
+    if (NI) IRCK(cudaMemcpyAsync(dtot.data(), tot_d, (size_t)NI * 8, cudaMemcpyDeviceToHost, st));
     IRCK(cudaFreeAsync(stats, st));
     IRCK(cudaStreamSynchronize(st));
+    if (replay) {
+        // every replayed total must be what the device computed; otherwise
+        // forget them and run again with a host round trip per level
+        bool same = rc == BEAST_OK || rc == BEAST_ERR_CAPACITY;
+        for (int k = 0; k < NI && same; ++k)
+            if (dtot[k] != ~0ull && ir->known_tot[k] != ~0ull && dtot[k] != ir->known_tot[k]) same = false;
+        if (!same) {
+            ir->known_pruned = -1;
+            ir->known_tot.clear();
+            return run(ir, st, out, capacity, written, visits, rejected, emit_last, false);
+        }
+    } else if (rc == BEAST_OK) {
+        if ((int)ir->known_tot.size() != NI) ir->known_tot.assign(NI, ~0ull);
+        for (int k = 0; k < NI; ++k)
+            if (step_tot[k] != ~0ull) ir->known_tot[k] = step_tot[k];
+        ir->known_trip.assign(trip.begin(), trip.begin() + NI);
+        ir->known_pruned = pruned;
+    }
     if (rc != BEAST_OK && rc != BEAST_ERR_CAPACITY) return rc;
     if (rc == BEAST_OK)   // learn each step's trip counts for the next run
         for (int i = 0; i < NI; ++i)

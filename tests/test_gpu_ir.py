@@ -150,3 +150,32 @@ def test_gemm_ir_tiny_kernel_shapes(beast, p, mode):
 def test_gemm_ir_medium_kernel_shapes(beast, mode):
     with _Env(mode):
         test_gemm_ir_medium_against_ir_oracle(beast)
+
+
+@pytest.mark.parametrize("which", ["tiny_D", "fuzz_11", "toy"])
+def test_replayed_runs_equal_first(beast, which):
+    """After its first run a handle enqueues every level without a host
+    round trip, sizing each level from the previous run's totals (checked at
+    the end): later counts and enumerations must equal the first and the
+    oracle's."""
+    if which == "toy":
+        spec = ir_specs.toy_specs()[sorted(ir_specs.toy_specs())[0]]
+        ref = oir.run(spec, records=True)
+        want = ref["records"]
+    else:
+        desc = bi.tiny("D") if which == "tiny_D" else bi.fuzz_space(11)
+        spec = ir_specs.gemm_spec(oracle.resolve(desc), desc["precision"])
+        ref = oracle.nest(desc, records=True)
+        want = None
+    with beast.IRSpace(spec) as sp:
+        first = sp.count()
+        for _ in range(3):
+            assert sp.count() == first
+            rec, st = sp.enumerate()
+            assert st == first
+            got = rec.cpu().numpy()
+            if want is not None:
+                assert np.array_equal(got, want)
+            else:
+                assert np.array_equal(pack(got), ref["records"].astype(np.uint64))
+    assert first["survivors"] == ref["survivors"] and first["visits"] == ref["visits"]
