@@ -43,6 +43,10 @@ for lv, nm in enumerate(["L1-L3", "L4", "L5-L7"]):
     print("   tile-ordered end times (us):", ["%.1f" % (e[i] / 1e3) for i in q])
     print("   look-back done (us) at tile quantiles:", ["%.1f" % (l[i] / 1e3) for i in q])
     print("   distinct CTAs %d, words max %d" % (len(set(t[:, 4] & 0xffffffff)), (t[:, 4] >> 32).max()))
+    idx = np.nonzero(m)[0]
+    for i in np.argsort(-e)[:4]:
+        print("   late tile %d: start %.2f counted %.2f looked back %.2f emitted %.2f us, words %d" % (
+            idx[i], s[i] / 1e3, c[i] / 1e3, l[i] / 1e3, e[i] / 1e3, t[i, 4] >> 32))
 for lv in range(3):
     t = tr[lv]
     for k in range(3):
